@@ -1,0 +1,365 @@
+#!/usr/bin/env python
+"""bench.py — iterated SpMV (power iteration) over BCCOO/BCCOO+ on B200, one JSON line.
+
+Workload (BASELINE.json configs[4], the config the metric "SpMV GFLOPS and achieved HBM
+GB/s at 1/2/4/8 B200" is quoted on; it fits one GPU): C5, a circuit/LP-like 50M x 50M
+matrix with ~1.0B non-zeros, fp32 (synth/c5gen.c).  A step is one power iteration:
+y_r = A_r x (fused BCCOO SpMV kernel, §3 of the paper), ||y||^2, scale, and for N > 1 the
+NCCL all-reduce of one scalar + all-gather of x.  The matrix is fixed as N grows
+(strong scaling); each rank builds only its nnz-balanced row block.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl yaspmv|reference]
+                  [--config c5|c4|c3-spheres|...] [--params '{"T":16,"C":256}']
+
+--impl reference times the CPU oracle (oracle/ref_csr.c, compensated CSR matvec with
+OpenMP) on a bounded row sample of the same workload — the slow baseline of this tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+# tuned defaults per config (yaspmv_tune on B200)
+DEFAULT_PARAMS = {
+    "c5": dict(h=1, w=1, S=1, T=16, C=256, col_mode=2),
+    "c4": dict(h=1, w=1, S=1, T=16, C=256),
+    "c3-spheres": dict(h=4, w=4, T=4, C=128),
+    "c3-cantilever": dict(h=4, w=4, T=4, C=128),
+    "c3-ship": dict(h=2, w=2, T=8, C=256),
+    "c2-f32": dict(h=4, w=4, T=4, C=128),
+    "c2-f64": dict(h=4, w=4, T=4, C=128),
+    "c1": dict(T=4, C=64),
+}
+
+
+def _env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+    FIELDS = ["clocks.sm", "clocks.max.sm", "clocks_event_reasons.sw_power_cap",
+              "clocks_event_reasons.hw_slowdown", "clocks_event_reasons.hw_thermal_slowdown",
+              "clocks_event_reasons.sw_thermal_slowdown"]
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), "--query-gpu=" + ",".join(self.FIELDS),
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+            return
+        self.t = threading.Thread(target=self._read, daemon=True)
+        self.t.start()
+        t0 = time.time()
+        while not self.rows and time.time() - t0 < 5:
+            time.sleep(0.02)
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == len(self.FIELDS):
+                self.rows.append(parts)
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.1)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        rows = self.rows
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        reasons = set()
+        for r in rows:
+            for name, v in zip(["sw_power_cap", "hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"], r[2:]):
+                if v.lower().startswith("active"):
+                    reasons.add(name)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(rows)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def load_matrix(config: str, rank: int, world: int, dtype):
+    """Returns (local CSR, layout) — the rank's nnz-balanced row block, columns remapped to
+    the padded all-gather space when world > 1."""
+    import synth
+    from synth import matrices as sm
+    from paper_conf_ppopp_yanlzz14_b200 import dist as D
+    if config == "c5":
+        if world == 1:
+            csr = sm.circuit_like_rows(0, 50_000_000, dtype=dtype)
+            L = D.Layout(0, 1, np.array([0, csr.m], dtype=np.int64), csr.m)
+            return csr, L
+        # global row lengths (cheap pass) -> partition -> generate only this rank's rows
+        import ctypes
+        P = sm.c5_params()
+        counts = np.empty(P.n, dtype=np.int64)
+        sm._lib().c5_count(ctypes.byref(P), ctypes.c_int64(0), ctypes.c_int64(P.n),
+                            counts.ctypes.data_as(ctypes.c_void_p))
+        rp = np.zeros(P.n + 1, dtype=np.int64)
+        np.cumsum(counts, out=rp[1:])
+        del counts
+        L = D.make_layout(rp, rank, world)
+        csr = sm.circuit_like_rows(L.r0, L.r1, dtype=dtype)
+    else:
+        full = synth.config_matrix(config)
+        if world == 1:
+            return full, D.Layout(0, 1, np.array([0, full.m], dtype=np.int64), full.m)
+        L = D.make_layout(full.row_ptr, rank, world)
+        csr = full.row_slice(L.r0, L.r1)
+    csr.col = D.remap_columns(csr.col, L.bounds, L.m_max)
+    csr.n = L.n_padded
+    return csr, L
+
+
+def run_reference(args, rank, world):
+    """The oracle (oracle/ref_csr.c) on a bounded row sample of the workload."""
+    if rank != 0:
+        return
+    from oracle import ref
+    import synth
+    from synth import matrices as sm
+    if args.config == "c5":
+        rows = 1 << 21  # 2M rows x ~20 nnz: ~0.3 s per oracle call on 16 cores
+        csr = sm.circuit_like_rows(0, rows, dtype=np.float32)
+        x = np.full(50_000_000, 1.0 / np.sqrt(5e7), dtype=np.float32)
+        sample = f"rows [0, {rows}) of C5 ({csr.nnz} nnz), all 50M columns"
+    else:
+        csr = synth.config_matrix(args.config)
+        x = synth.make_x(csr.n, csr.val.dtype, "uniform", 0)
+        sample = f"full {args.config} ({csr.nnz} nnz)"
+    for _ in range(args.warmup):
+        ref.spmv(csr.row_ptr, csr.col, csr.val, x, with_bound=False)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        ref.spmv(csr.row_ptr, csr.col, csr.val, x, with_bound=False)
+    dt = (time.perf_counter() - t0) / max(args.steps, 1)
+    gflops = 2.0 * csr.nnz / dt / 1e9
+    cores = ref.num_threads()
+    line = {"impl": "reference", "metric": "SpMV GFLOPS (power-iteration step)", "value": gflops, "unit": "GFLOPS",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32" if csr.val.dtype == np.float32 else "f64",
+            "data": "synthetic", "config": {"workload": args.config, "sample": sample},
+            "cpu_baseline": {"value": gflops, "unit": "GFLOPS", "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": gflops, "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(csr_full, x_np, budget_s=12.0):
+    """The oracle as it stands on the box's host cores, on a bounded row sample."""
+    from oracle import ref
+    m = csr_full.m
+    rows = min(m, 1 << 20)
+    while True:
+        sub = csr_full.row_slice(0, rows)
+        t0 = time.perf_counter()
+        ref.spmv(sub.row_ptr, sub.col, sub.val, x_np, with_bound=False)
+        dt = time.perf_counter() - t0
+        if dt > 0.5 or rows >= m:
+            break
+        rows = min(m, rows * 4)
+    reps = max(1, min(5, int(budget_s / max(dt, 1e-3))))
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        ref.spmv(sub.row_ptr, sub.col, sub.val, x_np, with_bound=False)
+        ts.append(time.perf_counter() - t0)
+    t = float(np.median(ts))
+    return {"value": 2.0 * sub.nnz / t / 1e9, "unit": "GFLOPS", "cores": ref.num_threads(), "kind": "oracle",
+            "sample": f"rows [0, {rows}) ({sub.nnz} nnz) of the workload, median of {reps}"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=400)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="yaspmv", choices=["yaspmv", "reference"])
+    ap.add_argument("--config", default="c5")
+    ap.add_argument("--params", default=None, help="JSON dict of build parameters")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    args = ap.parse_args()
+
+    world = _env_int("WORLD_SIZE", 1)
+    rank = _env_int("RANK", 0)
+    local_rank = _env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    from paper_conf_ppopp_yanlzz14_b200 import dist as D
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    dtype_np = np.float64 if args.config in ("c1", "c2-f64", "c3-ship-f64") else np.float32
+    tdt = torch.float64 if dtype_np == np.float64 else torch.float32
+
+    t_build0 = time.perf_counter()
+    csr, L = load_matrix(args.config, rank, world, dtype_np)
+    t_gen = time.perf_counter() - t_build0
+    params = dict(DEFAULT_PARAMS.get(args.config, {}))
+    if args.params:
+        params.update(json.loads(args.params))
+    big = csr.nnz > 50_000_000
+    params.setdefault("flags", 2 if big else 0)  # DROP_CSR for the 1B-nnz matrix
+    A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=local_rank, **params)
+    info = A.info()
+    t_build = time.perf_counter() - t_build0
+
+    ops = D.GpuOps(A, L.m_local, dev)
+    if args.config != "c5" and csr.m != csr.n and world == 1:
+        raise SystemExit("power iteration needs a square matrix")
+    pit = D.PowerIteration(L, ops, tdt, dev)
+    stream = torch.cuda.current_stream()
+
+    for _ in range(max(args.warmup, 3)):
+        pit.step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    # ---- timed region: K steps, CUDA events on the launching stream ----------------
+    sampler = ClockSampler(local_rank)
+    sampler.start()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e0.record(stream)
+    for k in range(args.steps):
+        # SpMV launches recorded separately: the dominant kernel's live duration
+        ev[k][0].record(stream)
+        ops.spmv(pit.x, pit.y[: L.m_local])
+        ev[k][1].record(stream)
+        ops.nrm2sq(pit.y[: L.m_local], pit.norm2)
+        if world > 1:
+            dist.all_reduce(pit.norm2)
+            ops.scale(pit.y[: L.m_local], pit.y[: L.m_local], pit.norm2)
+            dist.all_gather_into_tensor(pit.x, pit.y)
+        else:
+            ops.scale(pit.y[: L.m_local], pit.x[: L.m_local], pit.norm2)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    ms_total = e0.elapsed_time(e1)
+    spmv_ms = float(np.mean([a.elapsed_time(b) for a, b in ev]))
+    t = torch.tensor([ms_total, spmv_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_total, spmv_ms_max = float(t[0]), float(t[1])
+    ms_step = ms_total / args.steps
+
+    nnz_local = torch.tensor([float(info["nnz"])], dtype=torch.float64, device=dev)
+    alg_local = torch.tensor([float(info["alg_bytes"])], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(nnz_local)
+        dist.all_reduce(alg_local)
+    nnz_total = float(nnz_local.item())
+    gflops = 2.0 * nnz_total / (ms_step * 1e-3) / 1e9
+
+    # ---- e2e through the public API with HOST buffers (pinned) -----------------------
+    xh = torch.empty(L.n_padded, dtype=tdt).pin_memory()
+    xh.copy_(pit.x.cpu())
+    yh = torch.empty(L.m_local, dtype=tdt).pin_memory()
+    A.spmv_host(xh.numpy(), yh.numpy(), stream=stream.cuda_stream)
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(args.e2e_steps):
+        A.spmv_host(xh.numpy(), yh.numpy(), stream=stream.cuda_stream)
+    te = torch.tensor([(time.perf_counter() - t0) / args.e2e_steps], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_s = float(te.item())
+    e2e = {"value": 2.0 * nnz_total / e2e_s / 1e9, "unit": "GFLOPS",
+           "h2d_bytes_per_step": int(L.n_padded * np.dtype(dtype_np).itemsize * world),
+           "d2h_bytes_per_step": int(int(L.bounds[-1]) * np.dtype(dtype_np).itemsize),
+           "api": "yaspmv_spmv_host (pinned x in, y out, per rank)"}
+
+    if rank == 0:
+        peak, peak_kind = measured_peaks()
+        achieved = info["alg_bytes"] / (spmv_ms * 1e-3) / 1e9
+        traffic = None
+        prof = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.config}.json")
+        if os.path.exists(prof):
+            with open(prof) as f:
+                tr = json.load(f)
+            if tr.get("params") == info["params"] and world == 1:
+                traffic = tr.get("dram_bytes_per_launch")
+        line = {
+            "metric": "SpMV GFLOPS and achieved HBM GB/s (% of 8 TB/s)", "value": gflops, "unit": "GFLOPS",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f32" if dtype_np == np.float32 else "f64", "data": "synthetic",
+            "config": {"workload": args.config, "m": int(L.bounds[-1]), "nnz": int(nnz_total),
+                       "params": info["params"], "parallelism": f"row-partition x{world}, NCCL all-gather of x",
+                       "l2": "inputs larger than L2 (matrix 8.5 GB vs 126 MB L2), no flush" if args.config == "c5"
+                       else "L2-resident workload; back-to-back steps (warm L2)",
+                       "step": "y=A x (fused BCCOO SpMV) + ||y||^2 + scale" + (" + allreduce + allgather" if world > 1 else "")},
+            "spmv_ms": spmv_ms, "spmv_ms_max_over_ranks": spmv_ms_max,
+            "spmv_gflops": 2.0 * info["nnz"] / (spmv_ms * 1e-3) / 1e9,
+            "hbm_gbs_alg": achieved, "pct_of_8TBs": achieved / 8000.0 * 100.0,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                         "kernel": "spmv_bccoo_kernel" + (" + combine" if info["params"]["slices"] > 1 else ""),
+                         "alg_bytes_per_launch": info["alg_bytes"]},
+            "gpu_launches": (A.launches_per_spmv() + 3) * args.steps,
+            "clocks": clocks, "e2e": e2e,
+            "build": {"generate_s": t_gen, "build_s": t_build, "encode_upload_s": info["build_seconds"]},
+        }
+        if world == 1 and not args.no_cpu_baseline:
+            x_np = pit.x[: L.m_local].float().cpu().numpy().astype(dtype_np) if args.config == "c5" \
+                else pit.x.cpu().numpy()
+            if args.config == "c5":
+                line["cpu_baseline"] = cpu_baseline(csr, x_np)
+            else:
+                line["cpu_baseline"] = cpu_baseline(csr, x_np)
+        print(json.dumps(line), flush=True)
+    A.free()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,194 @@
+/* yaspmv.h — C ABI of the B200-native yaSpMV hot path: y = A·x over BCCOO / BCCOO+.
+ *
+ * The operation is the paper's problem statement, "sparse matrix vector multiplication"
+ * y = A·x (§1; §2.3), computed over the BCCOO format (§2.2,
+ * P:81-121) or its vertically sliced variant BCCOO+ (§2.3) by the
+ * matrix-based segmented sum of §3, with parameters chosen by the
+ * auto-tuner of §4 (Table 1).  The entry points are SURVEY.md §8(b).
+ *
+ * Conventions for every call
+ *   - extern "C", fixed-width integer types, plain host or device pointers; no C++ or
+ *     torch types cross this boundary.
+ *   - Return value is a yaspmv_status; on failure a message is available from
+ *     yaspmv_last_error() (thread-local, valid until the next call on that thread).
+ *   - "host" pointers are ordinary CPU memory (pageable or pinned); "device" pointers are
+ *     CUDA global memory of the handle's device (e.g. torch tensor .data_ptr()).
+ *   - Streams are cudaStream_t passed as void* (NULL = the legacy default stream).
+ *   - Matrix data types: YASPMV_F32 (float values, float x/y) or YASPMV_F64 (double).
+ *     Indices are int32 column indices and int64 row pointers.
+ *   - There is no CPU fallback: spmv-family calls on a host-only handle, or without a
+ *     CUDA device, fail with YASPMV_EINVAL / YASPMV_ECUDA.
+ */
+#ifndef YASPMV_H
+#define YASPMV_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct yaspmv_matrix_s* yaspmv_matrix; /* opaque; owns every encoded array */
+
+typedef enum {
+  YASPMV_OK = 0,
+  YASPMV_EINVAL = 1,       /* bad argument / index out of range / host-only handle     */
+  YASPMV_ENOMEM = 2,       /* host or device allocation failed                         */
+  YASPMV_ECUDA = 3,        /* CUDA runtime or launch error (message has the CUDA text) */
+  YASPMV_EUNSUPPORTED = 4  /* parameter combination with no compiled kernel            */
+} yaspmv_status;
+
+typedef enum { YASPMV_F32 = 0, YASPMV_F64 = 1 } yaspmv_dtype;
+
+/* Column-index storage (Table 1 "Col_index compress"). */
+enum { YASPMV_COL_AUTO = 0, YASPMV_COL_U16 = 1, YASPMV_COL_I32 = 2, YASPMV_COL_DELTA16 = 3 };
+/* Empty (stacked) block rows (reading Q1):
+ *   FILLER = one zero block per empty row (the paper's "multiple 1s"),
+ *   MAP    = seg_row map from row stops to rows + a zero-fill list. */
+enum { YASPMV_EMPTY_AUTO = 0, YASPMV_EMPTY_FILLER = 1, YASPMV_EMPTY_MAP = 2 };
+/* yaspmv_params.flags */
+enum {
+  YASPMV_KEEP_HOST = 1, /* keep the canonical host arrays for yaspmv_export              */
+  YASPMV_DROP_CSR = 2   /* free the normalised host CSR after upload (no tune/reencode)  */
+};
+
+/* Tunable parameters, Table 1.  0 in any field = auto/default. */
+typedef struct {
+  int32_t block_h;     /* h in {1,2,3,4}     (Table 1 "Block height")            */
+  int32_t block_w;     /* w in {1,2,4}       (Table 1 "Block width")             */
+  int32_t slices;      /* S >= 1; 1 = BCCOO, > 1 = BCCOO+ (P:307); S <= ceil(n/w) */
+  int32_t thread_tile; /* T in {4,8,16,32}: non-zero blocks per thread       */
+  int32_t cta_size;    /* C in {64,128,256,512}: threads per workgroup           */
+  int32_t col_mode;    /* YASPMV_COL_*; U16 requires ceil(n/w) < 65535           */
+  int32_t empty_mode;  /* YASPMV_EMPTY_*                                                  */
+  int32_t flags;       /* YASPMV_KEEP_HOST | YASPMV_DROP_CSR                             */
+} yaspmv_params;
+
+typedef struct {
+  int64_t m, n, nnz;         /* matrix shape and structural non-zeros after normalisation */
+  int64_t MB, NB, SW;        /* block rows, block columns, block columns per slice        */
+  int64_t nnzb;              /* stored blocks (incl. filler blocks), before padding       */
+  int64_t nnzb_pad;          /* padded to a multiple of T*C                       */
+  int64_t ntiles;            /* workgroup-level tiles = CTAs per SpMV launch              */
+  int64_t n_stops;           /* row stops ('0' bits)                               */
+  int64_t n_filler;          /* filler blocks (empty_mode FILLER)                         */
+  int64_t n_zero_rows;       /* zero-filled stacked rows (empty_mode MAP)                 */
+  int64_t format_bytes;      /* device bytes of the format read by one SpMV               */
+  int64_t alg_bytes;         /* algorithmic bytes per SpMV: format + x + y (+ 2*S*M tmp)  */
+  int64_t footprint_bytes;   /* Table-3 footprint: values + col + flag bits       */
+  yaspmv_params params;      /* resolved parameters (no zeros)                            */
+  int32_t dtype;             /* yaspmv_dtype                                               */
+  int32_t device;            /* CUDA device ordinal, -1 for a host-only handle            */
+  int32_t has_seg_row;       /* 1 if a seg_row map is stored                              */
+  int32_t regs_per_thread;   /* registers of the selected SpMV kernel (0 if host-only)    */
+  double build_seconds;      /* wall time of the last (re-)encode + upload                */
+  double tune_seconds;       /* wall time of the last yaspmv_tune                         */
+} yaspmv_info;
+
+/* ---------------------------------------------------------------- build / free
+ * yaspmv_build_csr: encode A (m x n, CSR) into BCCOO/BCCOO+ and upload it to `device`.
+ *   row_ptr: host, int64[m+1], row_ptr[0] = 0, non-decreasing (borrowed for the call).
+ *   col_idx: host, int32[nnz] in [0, n); rows may be unsorted and hold duplicates —
+ *            entries are stably sorted by column and duplicates summed in input order
+ *            (COO semantics); explicit zeros stay structural.
+ *   vals:    host, float or double [nnz] per `dtype`.
+ *   params:  NULL = defaults (h = w = S = 1, T = 16, C = 256, auto col / empty modes).
+ *   device:  CUDA device ordinal, or -1 for a HOST-ONLY handle (encode only: usable by
+ *            yaspmv_get_info / yaspmv_export, not by spmv).
+ *   out:     receives the new handle; the caller frees it with yaspmv_free.
+ * Errors: EINVAL (m, n < 0; NULL arrays with nnz > 0; index out of range; row_ptr not
+ * monotone; parameter outside Table 1's ranges; U16 with NB >= 65535; S > NB),
+ * ENOMEM, ECUDA, EUNSUPPORTED (no kernel compiled for (dtype, h, w, T, C)). */
+yaspmv_status yaspmv_build_csr(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                               const void* vals, yaspmv_dtype dtype, const yaspmv_params* params,
+                               int32_t device, yaspmv_matrix* out);
+
+/* yaspmv_build_coo: as build_csr from COO triples (row_idx, col_idx, vals)[nnz], any order,
+ * duplicates summed in input order (Q14). */
+yaspmv_status yaspmv_build_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row_idx,
+                               const int32_t* col_idx, const void* vals, yaspmv_dtype dtype,
+                               const yaspmv_params* params, int32_t device, yaspmv_matrix* out);
+
+/* yaspmv_free: releases every host and device array of A.  NULL-safe.  Must not be called
+ * while work using A is still pending on a stream (synchronize first). */
+void yaspmv_free(yaspmv_matrix A);
+
+/* ---------------------------------------------------------------- SpMV
+ * yaspmv_spmv: y := A·x  (overwrite; no alpha/beta).  Stream-ordered and asynchronous.
+ *   x: device, n elements of A's dtype, aligned to w * sizeof(value) bytes.
+ *   y: device, m elements; must not overlap x.
+ * Deterministic: the same handle and x give a bitwise identical y.  One handle must not
+ * run on two streams concurrently (it owns per-call scratch: ticket counter, carry
+ * status words, BCCOO+ partial-result buffer).  Empty rows give y = 0.
+ * Kernels: the fused SpMV (multiply, per-thread segmented sum, CTA segmented scan,
+ * decoupled look-back carries, write-back; §3) and, when S > 1, the slice
+ * combine. */
+yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream);
+
+/* yaspmv_spmv_host: y := A·x with HOST x / y: copies x host->device into handle-owned
+ * scratch, runs yaspmv_spmv, copies y device->host, and synchronizes `stream` before
+ * returning.  Pinned host memory gives full PCIe/NVLink-C2C bandwidth. */
+yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host, void* stream);
+
+/* ---------------------------------------------------------------- tuning (§4)
+ * yaspmv_tune: auto-tuner of PAPER.md §4: for the 4 block shapes with the
+ * smallest footprint it times the SpMV over thread tile T, CTA size C, slice count
+ * S and column mode on the device (scratch x/y owned by the tuner), then re-encodes A with
+ * the fastest parameters (ties within 1%: smaller footprint, then lexicographic).
+ * Re-encoding needs the normalised CSR the handle keeps unless built with
+ * YASPMV_DROP_CSR (then EINVAL).  On failure A keeps its previous parameters.
+ * `chosen` (nullable, host) receives the selected parameters. */
+yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen);
+
+/* yaspmv_reencode: re-encode A with new parameters (0 fields = keep current). */
+yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params);
+
+/* ---------------------------------------------------------------- introspection
+ * yaspmv_get_info: fills *out (host). */
+yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* out);
+
+/* Canonical (un-permuted) encoded arrays, SURVEY §8(c) E1-E9:
+ *  FLAGS      uint8 [nnzb_pad/8]  bit flags, 0 = row stop, LSB-first, pad bits 1
+ *  COL        uint16 [nnzb_pad] (COL_U16) or int32 [nnzb_pad] (I32 / DELTA16 escape array)
+ *  COL_DELTA  int16 [nnzb_pad]    segmented difference per thread tile, -1 = escape
+ *  VAL0..3    value array r [nnzb_pad*w] of A's dtype
+ *  SEG_ROW    int32 [n_stops]     stacked block row of each row stop (empty_mode MAP)
+ *  ZERO_ROWS  int32 [n_zero_rows] stacked block rows without blocks (empty_mode MAP)
+ *  CTA_SEG0   int32 [ntiles]      row stops before each workgroup tile
+ *  FRE        int32 [ntiles*C]    first-result entry of each thread (Fig. 6b) */
+enum {
+  YASPMV_ARR_FLAGS = 0, YASPMV_ARR_COL = 1, YASPMV_ARR_COL_DELTA = 2,
+  YASPMV_ARR_VAL0 = 3, YASPMV_ARR_VAL1 = 4, YASPMV_ARR_VAL2 = 5, YASPMV_ARR_VAL3 = 6,
+  YASPMV_ARR_SEG_ROW = 7, YASPMV_ARR_ZERO_ROWS = 8, YASPMV_ARR_CTA_SEG0 = 9, YASPMV_ARR_FRE = 10
+};
+
+/* yaspmv_export: copy canonical array `which` into host_dst (capacity `bytes`).  Returns
+ * the array's byte size in *nbytes (nullable).  host_dst may be NULL to query the size.
+ * Needs YASPMV_KEEP_HOST (or a host-only handle) except for CTA_SEG0 / FRE.
+ * yaspmv_export_device: the same array read back FROM THE DEVICE copy and un-permuted
+ * from the device layout (checks the uploaded arrays; device handles only). */
+yaspmv_status yaspmv_export(yaspmv_matrix A, int32_t which, void* host_dst, int64_t bytes, int64_t* nbytes);
+yaspmv_status yaspmv_export_device(yaspmv_matrix A, int32_t which, void* host_dst, int64_t bytes,
+                                   int64_t* nbytes);
+
+/* ---------------------------------------------------------------- power-iteration helpers
+ * yaspmv_nrm2sq: out_dev[0] (device double) := sum_i v[i]^2 over device v[n] of `dtype`,
+ *   accumulated in fp64, deterministic (fixed reduction tree).  scratch_dev: device,
+ *   >= yaspmv_nrm2sq_scratch_bytes(n) bytes, zero-initialised once by the caller.
+ * yaspmv_scale: dst[i] := src[i] / sqrt(norm2_dev[0]) (device; dst may equal src). */
+yaspmv_status yaspmv_nrm2sq(const void* v, int64_t n, yaspmv_dtype dtype, double* out_dev, void* scratch_dev,
+                            void* stream);
+int64_t yaspmv_nrm2sq_scratch_bytes(int64_t n);
+yaspmv_status yaspmv_scale(const void* src, void* dst, int64_t n, yaspmv_dtype dtype, const double* norm2_dev,
+                           void* stream);
+
+/* ---------------------------------------------------------------- misc */
+const char* yaspmv_last_error(void);
+const char* yaspmv_version(void);
+/* Kernel launches issued by the last yaspmv_spmv on this handle (1, or 2 with S > 1). */
+int32_t yaspmv_launches_per_spmv(yaspmv_matrix A);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* YASPMV_H */

@@ -1,0 +1,403 @@
+// capi.cpp — the C ABI of include/yaspmv.h: handles, upload to the device layout, SpMV
+// launch, export/introspection, the auto-tuner of PAPER.md §4, power-iteration helpers.
+#include <cuda_runtime.h>
+#include <omp.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <memory>
+#include <string>
+
+#include "handle.hpp"
+
+using namespace yaspmv;
+
+namespace yaspmv {
+static thread_local std::string g_err;
+void set_error(const std::string& msg) { g_err = msg; }
+yaspmv_status fail(yaspmv_status st, const std::string& msg) {
+  g_err = msg;
+  return st;
+}
+}  // namespace yaspmv
+
+#define CUDA_TRY(expr)                                                                       \
+  do {                                                                                       \
+    cudaError_t _e = (expr);                                                                 \
+    if (_e != cudaSuccess)                                                                   \
+      return fail(_e == cudaErrorMemoryAllocation ? YASPMV_ENOMEM : YASPMV_ECUDA,            \
+                  std::string(#expr) + ": " + cudaGetErrorString(_e));                       \
+  } while (0)
+
+namespace {
+
+double now_s() {
+  return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+Params from_abi(const yaspmv_params* p) {
+  Params q;
+  if (p) {
+    q.h = p->block_h;
+    q.w = p->block_w;
+    q.S = p->slices;
+    q.T = p->thread_tile;
+    q.C = p->cta_size;
+    q.col_mode = p->col_mode;
+    q.empty_mode = p->empty_mode;
+    q.flags = p->flags;
+  }
+  return q;
+}
+
+yaspmv_params to_abi(const Params& q) {
+  yaspmv_params p;
+  p.block_h = q.h;
+  p.block_w = q.w;
+  p.slices = q.S;
+  p.thread_tile = q.T;
+  p.cta_size = q.C;
+  p.col_mode = q.col_mode;
+  p.empty_mode = q.empty_mode;
+  p.flags = q.flags;
+  return p;
+}
+
+template <typename T>
+yaspmv_status upload(const T* src, size_t bytes, T** dst) {
+  *dst = nullptr;
+  if (bytes == 0) return YASPMV_OK;
+  CUDA_TRY(cudaMalloc((void**)dst, bytes));
+  CUDA_TRY(cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice));
+  return YASPMV_OK;
+}
+
+yaspmv_status upload_permuted(const uint8_t* src, int64_t ntiles, int C, int ptb, void** dst) {
+  *dst = nullptr;
+  const size_t bytes = (size_t)ntiles * C * ptb;
+  if (bytes == 0) return YASPMV_OK;
+  std::unique_ptr<uint8_t[]> tmp;
+  try {
+    tmp.reset(new uint8_t[bytes]);
+  } catch (const std::bad_alloc&) {
+    return fail(YASPMV_ENOMEM, "host staging allocation failed");
+  }
+  permute_to_device_layout(src, tmp.get(), ntiles, C, ptb);
+  CUDA_TRY(cudaMalloc(dst, bytes));
+  CUDA_TRY(cudaMemcpy(*dst, tmp.get(), bytes, cudaMemcpyHostToDevice));
+  return YASPMV_OK;
+}
+
+// Encoded host arrays -> a fresh set of device arrays in the device layout.
+yaspmv_status to_device_impl(const Canonical& c, int vsize, DevArrays& d, int64_t& n_escapes) {
+  const Params& p = c.p;
+  yaspmv_status st;
+  const int vptb = p.T * p.w * vsize;
+  for (int r = 0; r < p.h; ++r)
+    if ((st = upload_permuted(c.val[r].data(), c.ntiles, p.C, vptb, &d.val[r])) != YASPMV_OK) return st;
+  if (p.col_mode == COL_U16) {
+    st = upload_permuted(reinterpret_cast<const uint8_t*>(c.col16.data()), c.ntiles, p.C, 2 * p.T, &d.col);
+  } else if (p.col_mode == COL_I32) {
+    st = upload_permuted(reinterpret_cast<const uint8_t*>(c.col32.data()), c.ntiles, p.C, 4 * p.T, &d.col);
+  } else {
+    st = upload_permuted(reinterpret_cast<const uint8_t*>(c.delta.data()), c.ntiles, p.C, 2 * p.T, &d.col);
+    if (st == YASPMV_OK) st = upload(c.col32.data(), c.col32.size() * 4, &d.col32);
+  }
+  if (st != YASPMV_OK) return st;
+  if ((st = upload(c.flags.data(), c.flags.size(), &d.flags)) != YASPMV_OK) return st;
+  if ((st = upload(c.cta_seg0.data(), c.cta_seg0.size() * 4, &d.cta_seg0)) != YASPMV_OK) return st;
+  if ((st = upload(c.seg_row.data(), c.seg_row.size() * 4, &d.seg_row)) != YASPMV_OK) return st;
+  if ((st = upload(c.zero_rows.data(), c.zero_rows.size() * 4, &d.zero_rows)) != YASPMV_OK) return st;
+  CUDA_TRY(cudaMalloc((void**)&d.ticket, sizeof(unsigned long long)));
+  CUDA_TRY(cudaMemset(d.ticket, 0, sizeof(unsigned long long)));
+  const int64_t nt = std::max<int64_t>(c.ntiles, 1);
+  CUDA_TRY(cudaMalloc((void**)&d.status, nt * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMemset(d.status, 0, nt * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMalloc((void**)&d.carry, nt * p.h * sizeof(double)));
+  if (p.S > 1) CUDA_TRY(cudaMalloc(&d.tmp, (size_t)p.S * c.MB * p.h * vsize));
+  // escapes of the int16 delta column array (only they read col32)
+  n_escapes = 0;
+  if (p.col_mode == COL_DELTA)
+    for (int16_t v : c.delta) n_escapes += v == -1;
+  CUDA_TRY(cudaDeviceSynchronize());
+  return YASPMV_OK;
+}
+
+// Upload A->can; on success replace A's device arrays, on failure keep the old ones.
+yaspmv_status to_device(yaspmv_matrix A) {
+  CUDA_TRY(cudaSetDevice(A->device));
+  DevArrays nd;
+  int64_t esc = 0;
+  yaspmv_status st = to_device_impl(A->can, A->vsize, nd, esc);
+  if (st != YASPMV_OK) {
+    nd.free_all();
+    return st;
+  }
+  CUDA_TRY(cudaDeviceSynchronize());  // no launch may still use the old arrays
+  A->d.free_all();
+  A->d = nd;
+  A->n_escapes = esc;
+  return YASPMV_OK;
+}
+
+yaspmv_status select_kernel(yaspmv_matrix A) {
+  const Params& p = A->can.p;
+  if (A->device < 0) return YASPMV_OK;  // host-only handles never launch
+  A->kern = find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode);
+  if (!A->kern)
+    return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for dtype/h/w/T (values per thread exceed 512 bytes)");
+  if (A->device >= 0) {
+    int regs = 0, maxt = 0;
+    int e = A->kern->attr(&regs, &maxt);
+    if (e != 0) return fail(YASPMV_ECUDA, std::string("cudaFuncGetAttributes: ") + cudaGetErrorString((cudaError_t)e));
+    if (p.C > maxt) return fail(YASPMV_EUNSUPPORTED, "cta_size exceeds the kernel's launch bound");
+    A->regs = regs;
+  }
+  return YASPMV_OK;
+}
+
+// (re-)encode A->csr with params and upload; on failure A is left unchanged
+yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
+  const double t0 = now_s();
+  Params p;
+  yaspmv_status st = resolve_params(want, A->csr.m, A->csr.n, p);
+  if (st != YASPMV_OK) return st;
+  if (A->device >= 0 && !find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode))
+    return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for this (dtype, h, w, T): values per thread > 512 B");
+  Canonical c;
+  if ((st = encode(A->csr, p, c)) != YASPMV_OK) return st;
+  Canonical old;
+  std::swap(old, A->can);
+  A->can = std::move(c);
+  const KernelEntry* oldk = A->kern;
+  if ((st = select_kernel(A)) != YASPMV_OK) {
+    A->can = std::move(old);
+    A->kern = oldk;
+    return st;
+  }
+  if (A->device >= 0) {
+    if ((st = to_device(A)) != YASPMV_OK) {  // old device arrays are untouched
+      A->can = std::move(old);
+      A->kern = oldk;
+      return st;
+    }
+    if (!(p.flags & YASPMV_KEEP_HOST)) {
+      A->can.release_arrays();
+      A->have_host_arrays = false;
+    } else {
+      A->have_host_arrays = true;
+    }
+  } else {
+    A->have_host_arrays = true;
+  }
+  A->build_s = now_s() - t0;
+  return YASPMV_OK;
+}
+
+yaspmv_status build_common(yaspmv_matrix A, const Params& p) {
+  yaspmv_status st = encode_into(A, p);
+  if (st != YASPMV_OK) return st;
+  if (p.flags & YASPMV_DROP_CSR) {
+    A->csr = CSR();
+    A->have_csr = false;
+  } else {
+    A->csr.make_owned();
+    A->have_csr = true;
+  }
+  return YASPMV_OK;
+}
+
+yaspmv_status check_device(int32_t device) {
+  if (device < 0) return YASPMV_OK;
+  int n = 0;
+  cudaError_t e = cudaGetDeviceCount(&n);
+  if (e != cudaSuccess) return fail(YASPMV_ECUDA, std::string("no CUDA device: ") + cudaGetErrorString(e));
+  if (device >= n) return fail(YASPMV_EINVAL, "device ordinal out of range");
+  return YASPMV_OK;
+}
+
+int64_t format_bytes(const yaspmv_matrix A) {
+  const Canonical& c = A->can;
+  const Params& p = c.p;
+  int64_t b = c.nnzb_pad * (int64_t)p.h * p.w * A->vsize;       // values
+  b += c.nnzb_pad * (int64_t)col_bytes(p.col_mode);             // col / delta
+  b += A->n_escapes * 4;                                         // escape reads
+  b += c.nnzb_pad / 8;                                           // bit flags
+  b += c.ntiles * (4 + 8 + 8 * (int64_t)p.h);                    // cta_seg0, status, carry
+  if (c.has_seg_row) b += c.n_stops * 4;                         // seg_row
+  b += c.n_zero * 4;                                             // zero-fill list
+  return b;
+}
+
+int64_t alg_bytes(const yaspmv_matrix A) {
+  const Canonical& c = A->can;
+  const Params& p = c.p;
+  int64_t b = format_bytes(A) + c.n * A->vsize;  // + x
+  if (p.S == 1) b += c.m * A->vsize;             // + y
+  else b += (int64_t)p.S * c.MB * p.h * A->vsize + (int64_t)p.S * c.m * A->vsize + c.m * A->vsize;
+  return b;
+}
+
+yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
+  const Canonical& c = A->can;
+  const Params& p = c.p;
+  if (c.m == 0) return YASPMV_OK;
+  if (c.ntiles == 0) {
+    CUDA_TRY(cudaMemsetAsync(y, 0, (size_t)c.m * A->vsize, (cudaStream_t)stream));
+    return YASPMV_OK;
+  }
+  KArgs a;
+  for (int r = 0; r < 4; ++r) a.val[r] = A->d.val[r];
+  a.col = A->d.col;
+  a.col32 = A->d.col32;
+  a.flags = A->d.flags;
+  a.cta_seg0 = A->d.cta_seg0;
+  a.seg_row = A->d.seg_row;
+  a.zero_rows = A->d.zero_rows;
+  a.n_zero = c.n_zero;
+  a.x = x;
+  a.out = p.S == 1 ? y : A->d.tmp;
+  a.out_limit = p.S == 1 ? c.m : (int64_t)p.S * c.MB * p.h;
+  a.n = c.n;
+  a.ntiles = c.ntiles;
+  a.ticket = A->d.ticket;
+  a.status = A->d.status;
+  a.carry = A->d.carry;
+  A->kern->launch(a, p.C, c.ntiles, stream);
+  CUDA_TRY(cudaGetLastError());
+  if (p.S > 1) {
+    launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream);
+    CUDA_TRY(cudaGetLastError());
+  }
+  return YASPMV_OK;
+}
+
+}  // namespace
+
+// =====================================================================================
+extern "C" {
+
+const char* yaspmv_last_error(void) { return g_err.c_str(); }
+const char* yaspmv_version(void) { return "yaspmv-b200 0.1 (sm_100a)"; }
+
+yaspmv_status yaspmv_build_csr(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                               const void* vals, yaspmv_dtype dtype, const yaspmv_params* params,
+                               int32_t device, yaspmv_matrix* out) {
+  if (!out) return fail(YASPMV_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (dtype != YASPMV_F32 && dtype != YASPMV_F64) return fail(YASPMV_EINVAL, "bad dtype");
+  yaspmv_status st = check_device(device);
+  if (st != YASPMV_OK) return st;
+  std::unique_ptr<yaspmv_matrix_s> A(new (std::nothrow) yaspmv_matrix_s());
+  if (!A) return fail(YASPMV_ENOMEM, "handle allocation failed");
+  A->device = device;
+  A->dtype = dtype;
+  A->vsize = dtype == YASPMV_F32 ? 4 : 8;
+  if ((st = normalize_csr(m, n, row_ptr, col_idx, vals, A->vsize, A->csr)) != YASPMV_OK) return st;
+  if ((st = build_common(A.get(), from_abi(params))) != YASPMV_OK) return st;
+  *out = A.release();
+  return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_build_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row_idx, const int32_t* col_idx,
+                               const void* vals, yaspmv_dtype dtype, const yaspmv_params* params, int32_t device,
+                               yaspmv_matrix* out) {
+  if (!out) return fail(YASPMV_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (dtype != YASPMV_F32 && dtype != YASPMV_F64) return fail(YASPMV_EINVAL, "bad dtype");
+  yaspmv_status st = check_device(device);
+  if (st != YASPMV_OK) return st;
+  std::unique_ptr<yaspmv_matrix_s> A(new (std::nothrow) yaspmv_matrix_s());
+  if (!A) return fail(YASPMV_ENOMEM, "handle allocation failed");
+  A->device = device;
+  A->dtype = dtype;
+  A->vsize = dtype == YASPMV_F32 ? 4 : 8;
+  if ((st = normalize_coo(m, n, nnz, row_idx, col_idx, vals, A->vsize, A->csr)) != YASPMV_OK) return st;
+  if ((st = build_common(A.get(), from_abi(params))) != YASPMV_OK) return st;
+  *out = A.release();
+  return YASPMV_OK;
+}
+
+void yaspmv_free(yaspmv_matrix A) { delete A; }
+
+yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (!A->have_csr) return fail(YASPMV_EINVAL, "handle was built with YASPMV_DROP_CSR");
+  Params want = from_abi(params);
+  const Params& cur = A->can.p;
+  if (!want.h) want.h = cur.h;
+  if (!want.w) want.w = cur.w;
+  if (!want.S) want.S = cur.S;
+  if (!want.T) want.T = cur.T;
+  if (!want.C) want.C = cur.C;
+  if (!params) want.flags = cur.flags;
+  return encode_into(A, want);
+}
+
+yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle (built with device = -1): no CPU fallback");
+  if (A->can.m > 0 && !y) return fail(YASPMV_EINVAL, "y is NULL");
+  if (A->can.n > 0 && !x) return fail(YASPMV_EINVAL, "x is NULL");
+  const int64_t xb = A->can.n * A->vsize, yb = A->can.m * A->vsize;
+  const char* xc = static_cast<const char*>(x);
+  const char* yc = static_cast<const char*>(y);
+  if (xb > 0 && yb > 0 && xc < yc + yb && yc < xc + xb) return fail(YASPMV_EINVAL, "x and y overlap");
+  if (((uintptr_t)x) % ((uintptr_t)A->can.p.w * A->vsize) != 0)
+    return fail(YASPMV_EINVAL, "x must be aligned to w * sizeof(value) bytes");
+  return run_spmv(A, x, y, stream);
+}
+
+yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host, void* stream) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle: no CPU fallback");
+  const size_t xb = (size_t)A->can.n * A->vsize, yb = (size_t)A->can.m * A->vsize;
+  CUDA_TRY(cudaSetDevice(A->device));
+  if (!A->xs && xb) CUDA_TRY(cudaMalloc(&A->xs, xb));
+  if (!A->ys && yb) CUDA_TRY(cudaMalloc(&A->ys, yb));
+  cudaStream_t s = (cudaStream_t)stream;
+  if (xb) CUDA_TRY(cudaMemcpyAsync(A->xs, x_host, xb, cudaMemcpyHostToDevice, s));
+  yaspmv_status st = run_spmv(A, A->xs, A->ys, stream);
+  if (st != YASPMV_OK) return st;
+  if (yb) CUDA_TRY(cudaMemcpyAsync(y_host, A->ys, yb, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  return YASPMV_OK;
+}
+
+int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
+  if (!A || A->can.m == 0) return 0;
+  if (A->can.ntiles == 0) return 0;  // memset only
+  return A->can.p.S > 1 ? 2 : 1;
+}
+
+yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
+  if (!A || !o) return fail(YASPMV_EINVAL, "NULL argument");
+  const Canonical& c = A->can;
+  std::memset(o, 0, sizeof(*o));
+  o->m = c.m;
+  o->n = c.n;
+  o->nnz = c.nnz;
+  o->MB = c.MB;
+  o->NB = c.NB;
+  o->SW = c.SW;
+  o->nnzb = c.nnzb;
+  o->nnzb_pad = c.nnzb_pad;
+  o->ntiles = c.ntiles;
+  o->n_stops = c.n_stops;
+  o->n_filler = c.n_filler;
+  o->n_zero_rows = c.n_zero;
+  o->format_bytes = format_bytes(A);
+  o->alg_bytes = alg_bytes(A);
+  o->footprint_bytes = footprint_bytes(c.nnzb, c.p.h, c.p.w, A->vsize, col_bytes(c.p.col_mode));
+  o->params = to_abi(c.p);
+  o->dtype = A->dtype;
+  o->device = A->device;
+  o->has_seg_row = c.has_seg_row;
+  o->regs_per_thread = A->regs;
+  o->build_seconds = A->build_s;
+  o->tune_seconds = A->tune_s;
+  return YASPMV_OK;
+}
+
+}  // extern "C"

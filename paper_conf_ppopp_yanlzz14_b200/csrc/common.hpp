@@ -1,0 +1,117 @@
+// common.hpp — internal declarations shared by the encoder, kernels, tuner and C ABI.
+// Nothing here crosses the ABI (include/yaspmv.h is the boundary).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/yaspmv.h"
+
+namespace yaspmv {
+
+enum ColMode { COL_U16 = 1, COL_I32 = 2, COL_DELTA = 3 };
+enum EmptyMode { EMPTY_FILLER = 1, EMPTY_MAP = 2 };
+
+struct Params {
+  int h = 1, w = 1, S = 1, T = 16, C = 256, col_mode = 0, empty_mode = 0, flags = 0;
+};
+
+inline int col_bytes(int mode) { return mode == COL_I32 ? 4 : 2; }
+
+// Normalised CSR (sorted, distinct columns per row).  Either owns its arrays or views
+// the caller's (when the input already is normalised).
+struct CSR {
+  int64_t m = 0, n = 0, nnz = 0;
+  int vsize = 4;
+  const int64_t* rp = nullptr;
+  const int32_t* ci = nullptr;
+  const uint8_t* v = nullptr;
+  std::vector<int64_t> rp_own;
+  std::vector<int32_t> ci_own;
+  std::vector<uint8_t> v_own;
+  void adopt_owned() {
+    rp = rp_own.data();
+    ci = ci_own.data();
+    v = v_own.data();
+  }
+  void make_owned();  // copy a view into owned storage
+  bool owned() const { return rp == rp_own.data() && !rp_own.empty(); }
+};
+
+// Canonical BCCOO / BCCOO+ arrays, host side.
+struct Canonical {
+  int64_t m = 0, n = 0, nnz = 0, MB = 0, NB = 0, SW = 1;
+  int64_t nnzb = 0, nnzb_pad = 0, ntiles = 0, n_stops = 0, n_filler = 0;
+  int64_t n_zero = 0;   // zero-filled stacked rows (EMPTY_MAP)
+  int has_seg_row = 0;  // seg_row map present (EMPTY_MAP with empty rows)
+  Params p;
+  int vsize = 4;
+  std::vector<uint8_t> flags;     // nnzb_pad/8, LSB-first, 0 = row stop
+  std::vector<uint16_t> col16;    // COL_U16
+  std::vector<int32_t> col32;     // COL_I32, or the escape array of COL_DELTA
+  std::vector<int16_t> delta;     // COL_DELTA
+  std::vector<uint8_t> val[4];    // h arrays of nnzb_pad*w values (raw bytes)
+  std::vector<int32_t> seg_row;   // EMPTY_MAP with empty rows
+  std::vector<int32_t> zero_rows; // EMPTY_MAP with empty rows
+  std::vector<int32_t> cta_seg0;  // ntiles
+  void release_arrays();
+};
+
+// status helpers ------------------------------------------------------------------
+void set_error(const std::string& msg);
+yaspmv_status fail(yaspmv_status st, const std::string& msg);
+
+// encoder (encode.cpp) ---------------------------------------------------------------
+yaspmv_status normalize_csr(int64_t m, int64_t n, const int64_t* rp, const int32_t* ci, const void* v,
+                            int vsize, CSR& out);
+yaspmv_status normalize_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* ri, const int32_t* ci,
+                            const void* v, int vsize, CSR& out);
+yaspmv_status resolve_params(const Params& in, int64_t m, int64_t n, Params& out);
+yaspmv_status encode(const CSR& A, const Params& p, Canonical& out);
+// device layout: per workgroup tile, the per-thread byte runs (ptb bytes each) are
+// transposed into chunks of min(16, ptb) bytes so that chunk j of thread t lives at
+// (tile*C*nch + j*C + t) — the offline transpose of PAPER.md P:269-273.
+void permute_to_device_layout(const uint8_t* src, uint8_t* dst, int64_t ntiles, int C, int ptb);
+void permute_from_device_layout(const uint8_t* src, uint8_t* dst, int64_t ntiles, int C, int ptb);
+int64_t footprint_bytes(int64_t nnzb, int h, int w, int vsize, int s_c);
+int64_t count_blocks(const CSR& A, int h, int w);  // h x w blocks holding >= 1 entry (S = 1)
+
+// kernels (spmv_kernel.cuh / inst_*.cu / kernels_aux.cu) -----------------------------
+struct KArgs {
+  const void* val[4];
+  const void* col;         // device layout: u16 / i32 block columns or int16 deltas
+  const int32_t* col32;    // canonical int32 columns (escape path of COL_DELTA)
+  const uint8_t* flags;    // canonical packed bit flags
+  const int32_t* cta_seg0; // row stops before each tile
+  const int32_t* seg_row;  // nullable: stop -> stacked block row
+  const int32_t* zero_rows;
+  int64_t n_zero;
+  const void* x;
+  void* out;               // y (S == 1) or the BCCOO+ partial buffer tmp[S*MB*h]
+  int64_t out_limit;       // valid output elements
+  int64_t n;               // columns of A (x length)
+  int64_t ntiles;
+  unsigned long long* ticket;
+  unsigned long long* status;
+  double* carry;           // ntiles * h
+};
+
+typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
+typedef int (*AttrFn)(int* regs, int* max_threads);
+
+struct KernelEntry {
+  int dtype, h, w, T, cm;
+  LaunchFn launch;
+  AttrFn attr;
+};
+
+const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm);
+const std::vector<KernelEntry>& all_kernels();
+
+void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream);
+void launch_nrm2sq(const void* v, int64_t n, int dtype, double* out, double* partials, void* stream);
+int64_t nrm2sq_blocks(int64_t n);
+void launch_scale(const void* src, void* dst, int64_t n, int dtype, const double* norm2, void* stream);
+
+}  // namespace yaspmv

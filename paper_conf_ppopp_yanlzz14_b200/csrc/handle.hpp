@@ -1,0 +1,59 @@
+// handle.hpp — the opaque yaspmv_matrix handle (internal; not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "common.hpp"
+
+using yaspmv::CSR;
+using yaspmv::Canonical;
+using yaspmv::KernelEntry;
+
+struct DevArrays {
+  void* val[4] = {nullptr, nullptr, nullptr, nullptr};
+  void* col = nullptr;
+  int32_t* col32 = nullptr;
+  uint8_t* flags = nullptr;
+  int32_t* cta_seg0 = nullptr;
+  int32_t* seg_row = nullptr;
+  int32_t* zero_rows = nullptr;
+  unsigned long long* ticket = nullptr;
+  unsigned long long* status = nullptr;
+  double* carry = nullptr;
+  void* tmp = nullptr;
+  void free_all() {
+    void* ps[] = {val[0], val[1], val[2], val[3], col, col32, flags, cta_seg0, seg_row, zero_rows,
+                  ticket, status, carry, tmp};
+    for (void* p : ps)
+      if (p) cudaFree(p);
+    *this = DevArrays();
+  }
+};
+
+struct yaspmv_matrix_s {
+  int device = -1;
+  int dtype = 0;
+  int vsize = 4;
+  CSR csr;
+  bool have_csr = false;
+  Canonical can;
+  bool have_host_arrays = false;
+  DevArrays d;
+  const KernelEntry* kern = nullptr;
+  int regs = 0;
+  void* xs = nullptr;  // scratch for spmv_host
+  void* ys = nullptr;
+  int64_t n_escapes = 0;
+  double build_s = 0, tune_s = 0;
+  ~yaspmv_matrix_s() {
+    if (device >= 0) {
+      int cur = 0;
+      cudaGetDevice(&cur);
+      cudaSetDevice(device);
+      d.free_all();
+      if (xs) cudaFree(xs);
+      if (ys) cudaFree(ys);
+      cudaSetDevice(cur);
+    }
+  }
+};

@@ -1,0 +1,8 @@
+// Precompiled SpMV kernel instances: dtype double, block height 4, all block widths
+// {1,2,4} x thread tiles {4,8,16,32} x column modes (Table 1), restricted to
+// T*h*w*sizeof(value) <= 512 bytes of values per thread (register budget).
+#include "spmv_kernel.cuh"
+
+namespace yaspmv {
+void register_f64_h4(std::vector<KernelEntry>& R) { reg_h<double, 4>(R); }
+}  // namespace yaspmv

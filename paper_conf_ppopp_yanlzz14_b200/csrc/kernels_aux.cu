@@ -1,0 +1,147 @@
+// kernels_aux.cu — BCCOO+ slice combine, power-iteration helpers, and the
+// registry of precompiled SpMV instances.
+#include <cuda_runtime.h>
+
+#include <mutex>
+
+#include "common.hpp"
+
+namespace yaspmv {
+
+// ---------------------------------------------------------------- BCCOO+ combine
+// y[i] = sum_{s=0..S-1} tmp[s*stride + i], ascending s (Fig. 5; Q11), fp64
+// accumulation then one rounding.  Vectorised 4 elements per thread when aligned.
+template <typename VT>
+__global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, int64_t m, int64_t stride, int S) {
+  const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += nthreads) {
+    double s = (double)__ldcs(tmp + i);
+    for (int q = 1; q < S; ++q) s += (double)__ldcs(tmp + (int64_t)q * stride + i);
+    y[i] = (VT)s;
+  }
+}
+
+static int num_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
+
+void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream) {
+  if (m <= 0) return;
+  int64_t blocks = (m + 255) / 256;
+  const int64_t cap = (int64_t)num_sms() * 8;
+  if (blocks > cap) blocks = cap;
+  if (dtype == 0)
+    combine_kernel<float><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const float*)tmp, (float*)y, m, stride, S);
+  else
+    combine_kernel<double><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const double*)tmp, (double*)y, m, stride, S);
+}
+
+// ---------------------------------------------------------------- ||v||^2
+// Deterministic two-pass reduction: fixed grid, fixed per-block partials, one final block.
+static constexpr int NRM_THREADS = 256;
+static constexpr int NRM_MAX_BLOCKS = 1184;  // 8 x 148
+
+int64_t nrm2sq_blocks(int64_t n) {
+  int64_t b = (n + NRM_THREADS * 4 - 1) / (NRM_THREADS * 4);
+  if (b < 1) b = 1;
+  if (b > NRM_MAX_BLOCKS) b = NRM_MAX_BLOCKS;
+  return b;
+}
+
+__device__ __forceinline__ double block_sum(double v) {
+  __shared__ double sh[NRM_THREADS / 32];
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v;
+  __syncthreads();
+  double r = 0.0;
+  if (threadIdx.x == 0)
+    for (int q = 0; q < NRM_THREADS / 32; ++q) r += sh[q];
+  return r;
+}
+
+template <typename VT>
+__global__ void nrm2sq_partial(const VT* __restrict__ v, int64_t n, double* __restrict__ partials) {
+  double s = 0.0;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    const double a = (double)v[i];
+    s = fma(a, a, s);
+  }
+  s = block_sum(s);
+  if (threadIdx.x == 0) partials[blockIdx.x] = s;
+}
+
+__global__ void nrm2sq_final(const double* __restrict__ partials, int nb, double* __restrict__ out) {
+  double s = 0.0;
+  for (int i = threadIdx.x; i < nb; i += blockDim.x) s += partials[i];
+  s = block_sum(s);
+  if (threadIdx.x == 0) out[0] = s;
+}
+
+void launch_nrm2sq(const void* v, int64_t n, int dtype, double* out, double* partials, void* stream) {
+  const int64_t nb = nrm2sq_blocks(n);
+  cudaStream_t st = (cudaStream_t)stream;
+  if (dtype == 0) nrm2sq_partial<float><<<(unsigned)nb, NRM_THREADS, 0, st>>>((const float*)v, n, partials);
+  else nrm2sq_partial<double><<<(unsigned)nb, NRM_THREADS, 0, st>>>((const double*)v, n, partials);
+  nrm2sq_final<<<1, NRM_THREADS, 0, st>>>(partials, (int)nb, out);
+}
+
+// ---------------------------------------------------------------- dst = src / ||.||
+template <typename VT>
+__global__ void scale_kernel(const VT* src, VT* dst, int64_t n, const double* __restrict__ norm2) {
+  const double inv = 1.0 / sqrt(norm2[0]);
+  const VT f = (VT)inv;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) dst[i] = src[i] * f;
+}
+
+void launch_scale(const void* src, void* dst, int64_t n, int dtype, const double* norm2, void* stream) {
+  if (n <= 0) return;
+  int64_t blocks = (n + 255) / 256;
+  const int64_t cap = (int64_t)num_sms() * 8;
+  if (blocks > cap) blocks = cap;
+  cudaStream_t st = (cudaStream_t)stream;
+  if (dtype == 0) scale_kernel<float><<<(unsigned)blocks, 256, 0, st>>>((const float*)src, (float*)dst, n, norm2);
+  else scale_kernel<double><<<(unsigned)blocks, 256, 0, st>>>((const double*)src, (double*)dst, n, norm2);
+}
+
+// ---------------------------------------------------------------- registry
+void register_f32_h1(std::vector<KernelEntry>&);
+void register_f32_h2(std::vector<KernelEntry>&);
+void register_f32_h3(std::vector<KernelEntry>&);
+void register_f32_h4(std::vector<KernelEntry>&);
+void register_f64_h1(std::vector<KernelEntry>&);
+void register_f64_h2(std::vector<KernelEntry>&);
+void register_f64_h3(std::vector<KernelEntry>&);
+void register_f64_h4(std::vector<KernelEntry>&);
+
+const std::vector<KernelEntry>& all_kernels() {
+  static std::vector<KernelEntry> R;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    register_f32_h1(R);
+    register_f32_h2(R);
+    register_f32_h3(R);
+    register_f32_h4(R);
+    register_f64_h1(R);
+    register_f64_h2(R);
+    register_f64_h3(R);
+    register_f64_h4(R);
+  });
+  return R;
+}
+
+const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm) {
+  for (const KernelEntry& e : all_kernels())
+    if (e.dtype == dtype && e.h == h && e.w == w && e.T == T && e.cm == cm) return &e;
+  return nullptr;
+}
+
+}  // namespace yaspmv

@@ -1,0 +1,137 @@
+"""Multi-GPU iterated SpMV (power iteration) — one process per GPU, torch.distributed/NCCL.
+
+Not in the paper (single GPU); BASELINE.json north_star asks for it:
+  * rows are partitioned nnz-balanced into contiguous blocks, one per rank
+    (``nnz_balanced_bounds``); each rank encodes only its own row block (all N columns);
+  * x is replicated: every iteration all-gathers the ranks' y blocks into x over
+    NVLink/NVSwitch (NCCL ``all_gather_into_tensor``).  To use NCCL's equal-size path,
+    each rank's chunk is padded to m_max rows and column indices are remapped at build
+    time into that padded space (``remap_columns``); pad entries of x are never read;
+  * the normalisation needs one scalar all-reduce (sum of ||y_r||^2).
+
+The exchange logic is independent of where the local product runs: ``PowerIteration``
+takes an ``ops`` object (GPU kernels in the product; the CPU tests inject others to
+exercise the gloo path on world_size 2).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+
+def nnz_balanced_bounds(row_ptr: np.ndarray, P: int, h: int = 1) -> np.ndarray:
+    """b_r = lower_bound(row_ptr, r*nnz/P), rounded down to a multiple of h (block rows
+    never straddle ranks); b_0 = 0, b_P = m.  Ties go to the lower row."""
+    row_ptr = np.asarray(row_ptr, dtype=np.int64)
+    m = row_ptr.size - 1
+    nnz = int(row_ptr[-1])
+    b = np.zeros(P + 1, dtype=np.int64)
+    for r in range(1, P):
+        target = (r * nnz) // P
+        i = int(np.searchsorted(row_ptr, target, side="left"))
+        i = min(max(i, 0), m)
+        b[r] = (i // h) * h
+    b[P] = m
+    b = np.maximum.accumulate(b)
+    return b
+
+
+def remap_columns(col: np.ndarray, bounds: np.ndarray, m_max: int) -> np.ndarray:
+    """Column j (owned by rank r = the block with bounds[r] <= j < bounds[r+1]) moves to
+    r*m_max + (j - bounds[r]) in the padded, all-gathered x."""
+    col = np.asarray(col, dtype=np.int64)
+    r = np.searchsorted(bounds, col, side="right") - 1
+    return (r * m_max + (col - bounds[r])).astype(np.int32)
+
+
+def unpad(x_padded: np.ndarray, bounds: np.ndarray, m_max: int) -> np.ndarray:
+    P = bounds.size - 1
+    return np.concatenate([x_padded[r * m_max: r * m_max + (bounds[r + 1] - bounds[r])] for r in range(P)])
+
+
+@dataclass
+class Layout:
+    rank: int
+    world: int
+    bounds: np.ndarray
+    m_max: int
+
+    @property
+    def r0(self) -> int:
+        return int(self.bounds[self.rank])
+
+    @property
+    def r1(self) -> int:
+        return int(self.bounds[self.rank + 1])
+
+    @property
+    def m_local(self) -> int:
+        return self.r1 - self.r0
+
+    @property
+    def n_padded(self) -> int:
+        return self.world * self.m_max
+
+
+def make_layout(row_ptr: np.ndarray, rank: int, world: int, h: int = 1) -> Layout:
+    b = nnz_balanced_bounds(row_ptr, world, h)
+    m_max = int(np.max(np.diff(b))) if world > 0 else 0
+    return Layout(rank, world, b, max(m_max, 1))
+
+
+class GpuOps:
+    """Local steps on the GPU: the fused SpMV kernel(s) + ||y||^2 + scale (libyaspmv)."""
+
+    def __init__(self, A, n_local_rows: int, device):
+        import torch
+
+        from .matrix import nrm2sq_scratch_bytes
+        self.A = A
+        self.scratch = torch.zeros(nrm2sq_scratch_bytes(max(n_local_rows, 1)) // 8 + 1, dtype=torch.float64,
+                                   device=device)
+
+    def spmv(self, x, y):
+        self.A.spmv(x, y)
+
+    def nrm2sq(self, y, out):
+        from .matrix import nrm2sq
+        nrm2sq(y, out, self.scratch)
+
+    def scale(self, src, dst, norm2):
+        from .matrix import scale
+        scale(src, dst, norm2)
+
+    def launches_per_step(self) -> int:
+        return self.A.launches_per_spmv() + 3  # + nrm2sq (2) + scale (1)
+
+
+class PowerIteration:
+    """x_{k+1} = A x_k / ||A x_k|| with A row-partitioned over the process group."""
+
+    def __init__(self, layout: Layout, ops, dtype, device, group=None):
+        import torch
+        self.L = layout
+        self.ops = ops
+        self.group = group
+        self.x = torch.zeros(layout.n_padded, dtype=dtype, device=device)
+        self.y = torch.zeros(layout.m_max, dtype=dtype, device=device)   # padded local block
+        self.norm2 = torch.zeros(1, dtype=torch.float64, device=device)
+        n_true = int(layout.bounds[-1])
+        for r in range(layout.world):  # x_0 = 1/sqrt(N) on the real entries
+            a = r * layout.m_max
+            self.x[a: a + int(layout.bounds[r + 1] - layout.bounds[r])] = 1.0 / np.sqrt(max(n_true, 1))
+
+    def step(self):
+        import torch.distributed as dist
+        L = self.L
+        y_loc = self.y[: L.m_local]
+        self.ops.spmv(self.x, y_loc)                    # y_r = A_r x   (fused SpMV kernel)
+        self.ops.nrm2sq(y_loc, self.norm2)              # ||y_r||^2
+        if L.world > 1:
+            dist.all_reduce(self.norm2, group=self.group)          # 1 fp64 over NVLink
+            self.ops.scale(y_loc, y_loc, self.norm2)
+            dist.all_gather_into_tensor(self.x, self.y, group=self.group)  # replicate x
+        else:
+            self.ops.scale(y_loc, self.x[: L.m_local], self.norm2)
+        return self.x

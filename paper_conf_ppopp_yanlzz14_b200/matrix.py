@@ -1,0 +1,175 @@
+"""Python binding of the C ABI (include/yaspmv.h): argument marshalling only.
+
+Every step of the SpMV runs in libyaspmv.so (host encoder in C++, kernels in CUDA for
+sm_100a).  torch is used for device memory and streams only; numpy for host arrays.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _lib
+from ._lib import check, lib
+
+_DT = {np.dtype(np.float32): _lib.F32, np.dtype(np.float64): _lib.F64}
+
+
+def _ptr(a) -> int | None:
+    if a is None:
+        return None
+    if isinstance(a, int):
+        return a
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    return a.data_ptr()  # torch.Tensor
+
+
+def _stream(stream) -> int | None:
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def make_params(**kw) -> _lib.Params:
+    p = _lib.Params()
+    names = {"h": "block_h", "w": "block_w", "S": "slices", "T": "thread_tile", "C": "cta_size"}
+    for k, v in kw.items():
+        setattr(p, names.get(k, k), int(v))
+    return p
+
+
+class Matrix:
+    """A BCCOO / BCCOO+ encoded sparse matrix resident on one GPU (or host-only with
+    device=-1, for inspecting the encoder)."""
+
+    def __init__(self, handle: ctypes.c_void_p, dtype):
+        self._h = handle
+        self.dtype = np.dtype(dtype)
+
+    # ---------------------------------------------------------------- builders
+    @classmethod
+    def from_csr(cls, m: int, n: int, row_ptr, col, val, device: int = 0, **params) -> "Matrix":
+        row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+        col = np.ascontiguousarray(col, dtype=np.int32)
+        val = np.ascontiguousarray(val)
+        if val.dtype not in _DT:
+            raise TypeError("values must be float32 or float64")
+        h = ctypes.c_void_p()
+        p = make_params(**params)
+        check(lib.yaspmv_build_csr(m, n, row_ptr.ctypes.data, col.ctypes.data, val.ctypes.data, _DT[val.dtype],
+                                   ctypes.byref(p), device, ctypes.byref(h)))
+        return cls(h, val.dtype)
+
+    @classmethod
+    def from_coo(cls, m: int, n: int, rows, cols, vals, device: int = 0, **params) -> "Matrix":
+        rows = np.ascontiguousarray(rows, dtype=np.int32)
+        cols = np.ascontiguousarray(cols, dtype=np.int32)
+        vals = np.ascontiguousarray(vals)
+        h = ctypes.c_void_p()
+        p = make_params(**params)
+        check(lib.yaspmv_build_coo(m, n, rows.size, rows.ctypes.data, cols.ctypes.data, vals.ctypes.data,
+                                   _DT[vals.dtype], ctypes.byref(p), device, ctypes.byref(h)))
+        return cls(h, vals.dtype)
+
+    @classmethod
+    def from_synth(cls, csr, device: int = 0, **params) -> "Matrix":
+        return cls.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=device, **params)
+
+    # ---------------------------------------------------------------- lifetime
+    def free(self) -> None:
+        if self._h is not None and self._h.value:
+            lib.yaspmv_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.free()
+
+    # ---------------------------------------------------------------- compute
+    def spmv(self, x, y=None, stream=None):
+        """y := A·x for device tensors (torch) or raw device pointers; returns y."""
+        if y is None:
+            import torch
+            y = torch.empty(self.info()["m"], dtype=x.dtype, device=x.device)
+        check(lib.yaspmv_spmv(self._h, _ptr(x), _ptr(y), _stream(stream)))
+        return y
+
+    def spmv_host(self, x: np.ndarray, y: np.ndarray | None = None, stream=None) -> np.ndarray:
+        """y := A·x with host arrays (copies in and out inside the call)."""
+        x = np.ascontiguousarray(x, dtype=self.dtype)
+        if y is None:
+            y = np.empty(self.info()["m"], dtype=self.dtype)
+        check(lib.yaspmv_spmv_host(self._h, _ptr(x), _ptr(y), _stream(stream) if stream != 0 else 0))
+        return y
+
+    def tune(self, stream=None) -> dict:
+        p = _lib.Params()
+        check(lib.yaspmv_tune(self._h, _stream(stream), ctypes.byref(p)))
+        return p.as_dict()
+
+    def reencode(self, **params) -> None:
+        p = make_params(**params)
+        check(lib.yaspmv_reencode(self._h, ctypes.byref(p)))
+
+    # ---------------------------------------------------------------- introspection
+    def info(self) -> dict:
+        inf = _lib.Info()
+        check(lib.yaspmv_get_info(self._h, ctypes.byref(inf)))
+        return inf.as_dict()
+
+    def launches_per_spmv(self) -> int:
+        return int(lib.yaspmv_launches_per_spmv(self._h))
+
+    _ARR_DT = {"flags": np.uint8, "col_delta": np.int16, "seg_row": np.int32, "zero_rows": np.int32,
+               "cta_seg0": np.int32, "fre": np.int32}
+
+    def _arr_dtype(self, name: str):
+        if name.startswith("val"):
+            return self.dtype
+        if name == "col":
+            return np.uint16 if self.info()["params"]["col_mode"] == _lib.COL_U16 else np.int32
+        return self._ARR_DT[name]
+
+    def export(self, name: str, device: bool = False) -> np.ndarray:
+        """Canonical encoded array; device=True reads the uploaded
+        device copy and un-permutes it."""
+        fn = lib.yaspmv_export_device if device else lib.yaspmv_export
+        nb = ctypes.c_int64()
+        check(fn(self._h, _lib.ARR[name], None, 0, ctypes.byref(nb)))
+        out = np.empty(nb.value, dtype=np.uint8)
+        check(fn(self._h, _lib.ARR[name], out.ctypes.data if nb.value else None, nb.value, ctypes.byref(nb)))
+        return out.view(self._arr_dtype(name))
+
+
+def nrm2sq(v, out, scratch, stream=None) -> None:
+    """out[0] := sum v^2 (device, fp64, deterministic)."""
+    import torch
+    dt = _lib.F32 if v.dtype == torch.float32 else _lib.F64
+    check(lib.yaspmv_nrm2sq(v.data_ptr(), v.numel(), dt, out.data_ptr(), scratch.data_ptr(), _stream(stream)))
+
+
+def nrm2sq_scratch_bytes(n: int) -> int:
+    return int(lib.yaspmv_nrm2sq_scratch_bytes(n))
+
+
+def scale(src, dst, norm2, stream=None) -> None:
+    """dst := src / sqrt(norm2[0]) (device)."""
+    import torch
+    dt = _lib.F32 if src.dtype == torch.float32 else _lib.F64
+    check(lib.yaspmv_scale(src.data_ptr(), dst.data_ptr(), src.numel(), dt, norm2.data_ptr(), _stream(stream)))
+
+
+def version() -> str:
+    return lib.yaspmv_version().decode()
