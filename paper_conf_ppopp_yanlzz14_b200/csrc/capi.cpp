@@ -147,13 +147,16 @@ yaspmv_status select_kernel(yaspmv_matrix A) {
   A->kern = find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode);
   if (!A->kern)
     return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for dtype/h/w/T (values per thread exceed 512 bytes)");
-  if (A->device >= 0) {
-    int regs = 0, maxt = 0;
-    int e = A->kern->attr(&regs, &maxt);
-    if (e != 0) return fail(YASPMV_ECUDA, std::string("cudaFuncGetAttributes: ") + cudaGetErrorString((cudaError_t)e));
-    if (p.C > maxt) return fail(YASPMV_EUNSUPPORTED, "cta_size exceeds the kernel's launch bound");
-    A->regs = regs;
-  }
+  int regs = 0, maxt = 0, bps = 0;
+  int e = A->kern->attr(p.C, &regs, &maxt, &bps);
+  if (e != 0) return fail(YASPMV_ECUDA, std::string("kernel attributes: ") + cudaGetErrorString((cudaError_t)e));
+  if (p.C > maxt) return fail(YASPMV_EUNSUPPORTED, "cta_size exceeds the kernel's launch bound");
+  if (bps <= 0) return fail(YASPMV_EUNSUPPORTED, "kernel does not fit on an SM with this cta_size");
+  int sms = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, A->device);
+  // persistent CTAs: as many as are co-resident, never more than there are tiles
+  A->grid = std::max<int64_t>(1, std::min<int64_t>(A->can.ntiles, (int64_t)sms * bps));
+  A->regs = regs;
   return YASPMV_OK;
 }
 
@@ -261,10 +264,11 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
   a.out_limit = p.S == 1 ? c.m : (int64_t)p.S * c.MB * p.h;
   a.n = c.n;
   a.ntiles = c.ntiles;
+  a.period = c.ntiles + A->grid;
   a.ticket = A->d.ticket;
   a.status = A->d.status;
   a.carry = A->d.carry;
-  A->kern->launch(a, p.C, c.ntiles, stream);
+  A->kern->launch(a, p.C, A->grid, stream);
   CUDA_TRY(cudaGetLastError());
   if (p.S > 1) {
     launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream);

@@ -92,13 +92,14 @@ struct KArgs {
   int64_t out_limit;       // valid output elements
   int64_t n;               // columns of A (x length)
   int64_t ntiles;
+  int64_t period;          // tickets per launch = ntiles + grid (persistent CTAs)
   unsigned long long* ticket;
   unsigned long long* status;
   double* carry;           // ntiles * h
 };
 
 typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
-typedef int (*AttrFn)(int* regs, int* max_threads);
+typedef int (*AttrFn)(int C, int* regs, int* max_threads, int* blocks_per_sm);
 
 struct KernelEntry {
   int dtype, h, w, T, cm;

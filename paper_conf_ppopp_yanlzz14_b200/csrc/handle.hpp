@@ -41,6 +41,7 @@ struct yaspmv_matrix_s {
   DevArrays d;
   const KernelEntry* kern = nullptr;
   int regs = 0;
+  int64_t grid = 1;  // persistent CTAs per launch (fixed per encoding: ticket period)
   void* xs = nullptr;  // scratch for spmv_host
   void* ys = nullptr;
   int64_t n_escapes = 0;

@@ -48,7 +48,7 @@ def _dense_exact(csr, x):
 
 # ----------------------------------------------------------------------------- paper example
 @pytest.mark.parametrize("S", [1, 2])
-@pytest.mark.parametrize("T,C", [(4, 64), (16, 256), (32, 512)])
+@pytest.mark.parametrize("T,C", [(4, 64), (16, 256), (32, 256), (8, 512)])
 def test_paper_example_A(S, T, C):
     A = np.array([[0, 0, 1, 0, 0, 0, 2, 3], [0, 0, 4, 5, 0, 0, 6, 0],
                   [0, 0, 0, 0, 7, 8, 9, 10], [11, 12, 0, 0, 13, 14, 15, 16]], dtype=np.float32)
@@ -57,6 +57,16 @@ def test_paper_example_A(S, T, C):
     csr = synth.CSR(4, 8, rp, c.astype(np.int32), A[r, c])
     y, _ = _run(csr, np.arange(1, 9, dtype=np.float32), h=2, w=2, S=S, T=T, C=C)
     assert y.tolist() == [41, 74, 226, 417]          # Fig. 5
+
+
+def test_launch_bound_is_reported():
+    """2x2 fp32 blocks with T=32 hold 512 B of values per thread: compiled for C <= 256
+    only; C = 512 is refused with EUNSUPPORTED instead of failing at launch."""
+    from paper_conf_ppopp_yanlzz14_b200 import YaspmvError
+    csr = synth.random_tiny(1, m=8, n=8, density=0.5, dtype=np.float32)
+    with pytest.raises(YaspmvError) as e:
+        _run(csr, np.ones(8, np.float32), h=2, w=2, T=32, C=512)
+    assert e.value.status == 4
 
 
 # ----------------------------------------------------------------------------- brute force grid
