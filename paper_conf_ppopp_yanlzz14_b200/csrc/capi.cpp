@@ -8,6 +8,7 @@
 #include <cstring>
 #include <memory>
 #include <string>
+#include <cstdlib>
 
 #include "handle.hpp"
 
@@ -154,8 +155,9 @@ yaspmv_status select_kernel(yaspmv_matrix A) {
   if (bps <= 0) return fail(YASPMV_EUNSUPPORTED, "kernel does not fit on an SM with this cta_size");
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, A->device);
-  // persistent CTAs: as many as are co-resident, never more than there are tiles
-  A->grid = std::max<int64_t>(1, std::min<int64_t>(A->can.ntiles, (int64_t)sms * bps));
+  // one CTA per workgroup-level tile (ticketed)
+  A->grid = std::max<int64_t>(1, A->can.ntiles);
+  (void)sms;
   A->regs = regs;
   return YASPMV_OK;
 }
@@ -264,7 +266,7 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
   a.out_limit = p.S == 1 ? c.m : (int64_t)p.S * c.MB * p.h;
   a.n = c.n;
   a.ntiles = c.ntiles;
-  a.period = c.ntiles + A->grid;
+  a.period = c.ntiles;
   a.ticket = A->d.ticket;
   a.status = A->d.status;
   a.carry = A->d.carry;
