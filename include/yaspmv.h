@@ -83,6 +83,8 @@ typedef struct {
   int32_t regs_per_thread;   /* registers of the selected SpMV kernel (0 if host-only)    */
   double build_seconds;      /* wall time of the last (re-)encode + upload                */
   double tune_seconds;       /* wall time of the last yaspmv_tune                         */
+  int32_t tune_candidates;   /* candidates timed by the last yaspmv_tune                   */
+  int32_t reserved;
 } yaspmv_info;
 
 /* ---------------------------------------------------------------- build / free

@@ -9,7 +9,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libyaspmv.so")
+# YASPMV_LIB_PATH: development override (A/B builds of the same sources); default in-tree
+LIB_PATH = os.environ.get("YASPMV_LIB_PATH") or os.path.join(_HERE, "libyaspmv.so")
 
 # status codes / enums (yaspmv.h)
 OK, EINVAL, ENOMEM, ECUDA, EUNSUPPORTED = 0, 1, 2, 3, 4
@@ -44,7 +45,8 @@ class Info(ctypes.Structure):
                 ("format_bytes", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("footprint_bytes", ctypes.c_int64), ("params", Params), ("dtype", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("has_seg_row", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
-                ("build_seconds", ctypes.c_double), ("tune_seconds", ctypes.c_double)]
+                ("build_seconds", ctypes.c_double), ("tune_seconds", ctypes.c_double),
+                ("tune_candidates", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
     def as_dict(self):
         d = {}

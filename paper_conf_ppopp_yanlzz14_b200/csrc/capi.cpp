@@ -162,6 +162,40 @@ yaspmv_status select_kernel(yaspmv_matrix A) {
   return YASPMV_OK;
 }
 
+// Make `c` A's encoding: select the kernel, upload, release host arrays unless kept.
+// On failure A keeps its previous encoding (host and device).
+yaspmv_status install_canonical_impl(yaspmv_matrix A, Canonical&& c, int flags) {
+  Canonical old;
+  std::swap(old, A->can);
+  A->can = std::move(c);
+  const KernelEntry* oldk = A->kern;
+  const int64_t oldgrid = A->grid;
+  yaspmv_status st;
+  if ((st = select_kernel(A)) != YASPMV_OK) {
+    A->can = std::move(old);
+    A->kern = oldk;
+    A->grid = oldgrid;
+    return st;
+  }
+  if (A->device >= 0) {
+    if ((st = to_device(A)) != YASPMV_OK) {  // old device arrays are untouched
+      A->can = std::move(old);
+      A->kern = oldk;
+      A->grid = oldgrid;
+      return st;
+    }
+    if (!(flags & YASPMV_KEEP_HOST)) {
+      A->can.release_arrays();
+      A->have_host_arrays = false;
+    } else {
+      A->have_host_arrays = true;
+    }
+  } else {
+    A->have_host_arrays = true;
+  }
+  return YASPMV_OK;
+}
+
 // (re-)encode A->csr with params and upload; on failure A is left unchanged
 yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
   const double t0 = now_s();
@@ -172,30 +206,7 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
     return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for this (dtype, h, w, T): values per thread > 512 B");
   Canonical c;
   if ((st = encode(A->csr, p, c)) != YASPMV_OK) return st;
-  Canonical old;
-  std::swap(old, A->can);
-  A->can = std::move(c);
-  const KernelEntry* oldk = A->kern;
-  if ((st = select_kernel(A)) != YASPMV_OK) {
-    A->can = std::move(old);
-    A->kern = oldk;
-    return st;
-  }
-  if (A->device >= 0) {
-    if ((st = to_device(A)) != YASPMV_OK) {  // old device arrays are untouched
-      A->can = std::move(old);
-      A->kern = oldk;
-      return st;
-    }
-    if (!(p.flags & YASPMV_KEEP_HOST)) {
-      A->can.release_arrays();
-      A->have_host_arrays = false;
-    } else {
-      A->have_host_arrays = true;
-    }
-  } else {
-    A->have_host_arrays = true;
-  }
+  if ((st = install_canonical_impl(A, std::move(c), p.flags)) != YASPMV_OK) return st;
   A->build_s = now_s() - t0;
   return YASPMV_OK;
 }
@@ -280,6 +291,10 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
 }
 
 }  // namespace
+
+yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags) {
+  return install_canonical_impl(A, std::move(c), flags);
+}
 
 // =====================================================================================
 extern "C" {
@@ -403,6 +418,7 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
   o->regs_per_thread = A->regs;
   o->build_seconds = A->build_s;
   o->tune_seconds = A->tune_s;
+  o->tune_candidates = A->tune_candidates;
   return YASPMV_OK;
 }
 

@@ -228,19 +228,24 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
     if (NB >= 65535) cms.push_back(COL_DELTA);
     for (int S : Ss) {
       if (S > std::max<int64_t>(NB, 1)) continue;
-      for (int cm : cms)
+      for (int cm : cms) {
+        // one encode per (h, w, S, col mode) at the largest tile; (T, C) variants derive
+        Params bp0;
+        bp0.h = sh.h; bp0.w = sh.w; bp0.S = S; bp0.T = 32; bp0.C = 512; bp0.col_mode = cm;
+        bp0.empty_mode = saved.empty_mode;
+        Params rp;
+        if (resolve_params(bp0, M.m, M.n, rp) != YASPMV_OK) continue;
+        Canonical base;
+        if (encode(M, rp, base) != YASPMV_OK) continue;
         for (int T : {4, 8, 16, 32}) {
           if (!find_kernel(A->dtype, sh.h, sh.w, T, cm)) continue;
           for (int C : {64, 128, 256, 512}) {
-            // occupancy bound: at least 2 tiles per SM unless the matrix is tiny
-            const int64_t nnzb_est = (int64_t)(sh.fp / std::max(1, sh.h * sh.w * vs));
-            const int64_t tiles = (nnzb_est + (int64_t)T * C - 1) / ((int64_t)T * C);
-            if (tiles < 2 * sms && (T * C) > 256 * 4) continue;
-            Params p;
-            p.h = sh.h; p.w = sh.w; p.S = S; p.T = T; p.C = C; p.col_mode = cm; p.empty_mode = saved.empty_mode;
-            p.flags = 0;
-            yaspmv_params ap{p.h, p.w, p.S, p.T, p.C, p.col_mode, p.empty_mode, 0};
-            if (yaspmv_reencode(A, &ap) != YASPMV_OK) continue;  // e.g. C above the launch bound
+            // occupancy bound: at least 2 tiles per SM unless the tile is small
+            const int64_t tiles = (base.nnzb + (int64_t)T * C - 1) / ((int64_t)T * C);
+            if (tiles < 2 * sms && (T * C) > 1024) continue;
+            Canonical cand;
+            if (derive_tc(base, T, C, cand) != YASPMV_OK) continue;
+            if (install_canonical(A, std::move(cand), 0) != YASPMV_OK) continue;  // e.g. launch bound
             bool ok = true;
             for (int it = 0; it < 3 && ok; ++it) ok = yaspmv_spmv(A, x, y, stream) == YASPMV_OK;
             if (!ok) continue;
@@ -260,6 +265,7 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
             results.push_back({ts[ts.size() / 2], info.format_bytes, A->can.p});
           }
         }
+      }
     }
   }
   cudaEventDestroy(e0);
@@ -286,6 +292,7 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
   yaspmv_status rs = yaspmv_reencode(A, &bp);
   if (rs != YASPMV_OK) return rs;
   A->tune_s = now_s() - t0;
+  A->tune_candidates = (int)results.size();
   if (chosen) {
     const Params& q = A->can.p;
     *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags};

@@ -69,6 +69,7 @@ yaspmv_status normalize_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* ri
                             const void* v, int vsize, CSR& out);
 yaspmv_status resolve_params(const Params& in, int64_t m, int64_t n, Params& out);
 yaspmv_status encode(const CSR& A, const Params& p, Canonical& out);
+yaspmv_status derive_tc(const Canonical& base, int T, int C, Canonical& out);
 // device layout: per workgroup tile, the per-thread byte runs (ptb bytes each) are
 // transposed into chunks of min(16, ptb) bytes so that chunk j of thread t lives at
 // (tile*C*nch + j*C + t) — the offline transpose of PAPER.md P:269-273.

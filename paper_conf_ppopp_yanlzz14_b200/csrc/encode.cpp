@@ -399,6 +399,54 @@ yaspmv_status encode(const CSR& A, const Params& p, Canonical& out) {
   return YASPMV_OK;
 }
 
+// ------------------------------------------------------------------------- tuner helper
+// The canonical arrays of the same (h, w, S, col mode) for another (T, C): T*C divides the
+// base tile, so the arrays are prefixes of the base ones (padding has the same content),
+// except the per-thread delta array and the per-tile stop counts, which are recomputed.
+yaspmv_status derive_tc(const Canonical& base, int T, int C, Canonical& out) {
+  const int64_t TC = (int64_t)T * C, BTC = (int64_t)base.p.T * base.p.C;
+  if (BTC % TC != 0) return fail(YASPMV_EINVAL, "derive_tc: tile does not divide the base tile");
+  out = Canonical();
+  out.m = base.m; out.n = base.n; out.nnz = base.nnz; out.MB = base.MB; out.NB = base.NB; out.SW = base.SW;
+  out.nnzb = base.nnzb; out.n_stops = base.n_stops; out.n_filler = base.n_filler; out.n_zero = base.n_zero;
+  out.has_seg_row = base.has_seg_row; out.vsize = base.vsize;
+  out.p = base.p;
+  out.p.T = T;
+  out.p.C = C;
+  out.nnzb_pad = (out.nnzb + TC - 1) / TC * TC;
+  out.ntiles = out.nnzb_pad / TC;
+  const int64_t NP = out.nnzb_pad;
+  const int w = base.p.w, vs = base.vsize;
+  try {
+    out.flags.assign(base.flags.begin(), base.flags.begin() + NP / 8);
+    if (!base.col16.empty()) out.col16.assign(base.col16.begin(), base.col16.begin() + NP);
+    if (!base.col32.empty()) out.col32.assign(base.col32.begin(), base.col32.begin() + NP);
+    for (int r = 0; r < base.p.h; ++r) out.val[r].assign(base.val[r].begin(), base.val[r].begin() + (size_t)NP * w * vs);
+    out.seg_row = base.seg_row;
+    out.zero_rows = base.zero_rows;
+    if (base.p.col_mode == COL_DELTA) {
+      out.delta.resize(NP);
+#pragma omp parallel for schedule(static)
+      for (int64_t b = 0; b < NP; ++b) {
+        const int64_t prev = (b % T == 0) ? 0 : out.col32[b - 1];
+        const int64_t d = (int64_t)out.col32[b] - prev;
+        out.delta[b] = (d < -32768 || d > 32767 || d == -1) ? (int16_t)-1 : (int16_t)d;
+      }
+    }
+    out.cta_seg0.assign(out.ntiles, 0);
+    int64_t acc = 0;
+    const int64_t tb = TC / 8;
+    for (int64_t k = 0; k < out.ntiles; ++k) {
+      out.cta_seg0[k] = (int32_t)acc;
+      for (int64_t q = 0; q < tb; ++q) acc += 8 - __builtin_popcount(out.flags[k * tb + q]);
+    }
+  } catch (const std::bad_alloc&) {
+    out = Canonical();
+    return fail(YASPMV_ENOMEM, "host allocation failed in derive_tc");
+  }
+  return YASPMV_OK;
+}
+
 // ------------------------------------------------------------------------- layout
 void permute_to_device_layout(const uint8_t* src, uint8_t* dst, int64_t ntiles, int C, int ptb) {
   const int ch = ptb < 16 ? ptb : 16, nch = ptb / ch;

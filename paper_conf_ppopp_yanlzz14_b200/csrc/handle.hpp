@@ -46,6 +46,7 @@ struct yaspmv_matrix_s {
   void* ys = nullptr;
   int64_t n_escapes = 0;
   double build_s = 0, tune_s = 0;
+  int tune_candidates = 0;
   ~yaspmv_matrix_s() {
     if (device >= 0) {
       int cur = 0;
@@ -58,3 +59,6 @@ struct yaspmv_matrix_s {
     }
   }
 };
+
+// capi.cpp: make an already encoded Canonical the handle's encoding (kernel + upload)
+yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags);

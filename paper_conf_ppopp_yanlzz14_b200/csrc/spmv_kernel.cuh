@@ -389,8 +389,11 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
 }
 
 // One CTA per workgroup-level tile; logical tile ids from an atomic ticket.
+#ifndef YASPMV_MINB
+#define YASPMV_MINB 1
+#endif
 template <typename VT, int H, int W, int T, int CM>
-__global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC) spmv_bccoo_kernel(const KArgs a) {
+__global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) spmv_bccoo_kernel(const KArgs a) {
   __shared__ ScanShared<VT, H> sh;
   if (threadIdx.x == 0) {
     const unsigned long long tk = atomicAdd(a.ticket, 1ull);

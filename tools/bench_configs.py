@@ -1,0 +1,94 @@
+"""Per-config SpMV measurements (BASELINE.json configs C1-C4; C5 is bench.py's workload):
+auto-tuned parameters (yaspmv_tune, §4), SpMV time warm (L2-resident, back-to-back) and
+cold (a 2x-L2 scratch write between launches), GFLOPS, algorithmic GB/s and fraction of
+the measured HBM peak, parity against the oracle, and the oracle's own CPU time.
+One JSON line per config; --md writes a markdown table.
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+CONFIGS = ["c1", "c2-f32", "c2-f64", "c3-spheres", "c3-cantilever", "c3-ship", "c3-ship-f64", "c4"]
+
+
+def timed(fn, iters, flush=None):
+    import torch
+    ts = []
+    for _ in range(iters):
+        if flush is not None:
+            flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    return float(np.median(ts))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--configs", default=",".join(CONFIGS))
+    ap.add_argument("--iters", type=int, default=50)
+    ap.add_argument("--md", default=None)
+    args = ap.parse_args()
+    import torch
+
+    import synth
+    from oracle import ref
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
+    l2 = torch.cuda.get_device_properties(0).L2_cache_size
+    flush = torch.empty(2 * l2, dtype=torch.uint8, device="cuda")
+    rows = []
+    for name in args.configs.split(","):
+        csr = synth.config_matrix(name)
+        dt = csr.val.dtype
+        x_np = synth.make_x(csr.n, dt, "unit" if name == "c4" else "uniform", 3)
+        x = torch.from_numpy(x_np).cuda()
+        y = torch.empty(csr.m, dtype=x.dtype, device="cuda")
+        y_ref, bound = ref.spmv(csr.row_ptr, csr.col, csr.val, x_np)
+        t0 = time.perf_counter()
+        ref.spmv(csr.row_ptr, csr.col, csr.val, x_np, with_bound=False)
+        t_cpu = time.perf_counter() - t0
+        A = Matrix.from_synth(csr, device=0)
+        chosen = A.tune()
+        info = A.info()
+        for _ in range(5):
+            A.spmv(x, y)
+        warm = timed(lambda: A.spmv(x, y), args.iters)
+        cold = timed(lambda: A.spmv(x, y), max(10, args.iters // 5), flush)
+        ok, worst = ref.check_tolerance(y.cpu().numpy(), y_ref, bound, dt)
+        r = {"config": name, "m": csr.m, "nnz": csr.nnz, "dtype": str(dt), "params": chosen,
+             "tune_s": info["tune_seconds"], "tune_candidates": info["tune_candidates"],
+             "ms_warm": warm, "ms_cold": cold,
+             "gflops_warm": 2 * csr.nnz / warm / 1e6, "gflops_cold": 2 * csr.nnz / cold / 1e6,
+             "alg_bytes": info["alg_bytes"], "alg_GBs_cold": info["alg_bytes"] / cold / 1e6,
+             "frac_of_measured_hbm_cold": info["alg_bytes"] / cold / 1e6 / peak,
+             "footprint_MB": info["footprint_bytes"] / 1e6, "parity_ok": ok, "worst_err_over_tol": worst,
+             "oracle_cpu_ms": t_cpu * 1e3, "oracle_threads": ref.num_threads()}
+        print(json.dumps(r), flush=True)
+        rows.append(r)
+        A.free()
+    if args.md:
+        with open(args.md, "w") as f:
+            f.write("| config | nnz | dtype | tuned (h,w,T,C,S,col) | tune s | warm ms | cold ms | GFLOPS (cold) | alg GB/s (cold) | frac of measured HBM | parity (worst err/tol) | oracle CPU ms |\n")
+            f.write("|---|---|---|---|---|---|---|---|---|---|---|---|\n")
+            for r in rows:
+                p = r["params"]
+                f.write(f"| {r['config']} | {r['nnz']:,} | {r['dtype']} | {p['block_h']}x{p['block_w']}, T={p['thread_tile']}, "
+                        f"C={p['cta_size']}, S={p['slices']}, col={p['col_mode']} | {r['tune_s']:.1f} | {r['ms_warm']:.4f} | "
+                        f"{r['ms_cold']:.4f} | {r['gflops_cold']:.1f} | {r['alg_GBs_cold']:.0f} | {r['frac_of_measured_hbm_cold']:.3f} | "
+                        f"{'ok' if r['parity_ok'] else 'FAIL'} ({r['worst_err_over_tol']:.2g}) | {r['oracle_cpu_ms']:.2f} |\n")
+
+
+if __name__ == "__main__":
+    main()
