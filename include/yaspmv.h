@@ -132,6 +132,15 @@ yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream)
  * returning.  Pinned host memory gives full PCIe/NVLink-C2C bandwidth. */
 yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host, void* stream);
 
+/* yaspmv_spmv_host_async: y := A·x with HOST x / y, returning before completion.  Calls on
+ * one handle overlap the host->device copy of call k+1, the SpMV of call k and the
+ * device->host copy of call k-1 (two handle-owned device buffer pairs, two internal copy
+ * streams, events chaining them to `stream`).  x_host must stay unchanged and y_host valid
+ * until yaspmv_host_sync(A); pinned host memory is needed for the copies to overlap.
+ * yaspmv_host_sync: waits for every outstanding yaspmv_spmv_host_async of the handle. */
+yaspmv_status yaspmv_spmv_host_async(yaspmv_matrix A, const void* x_host, void* y_host, void* stream);
+yaspmv_status yaspmv_host_sync(yaspmv_matrix A);
+
 /* ---------------------------------------------------------------- tuning (§4)
  * yaspmv_tune: auto-tuner of PAPER.md §4: for the 4 block shapes with the
  * smallest footprint it times the SpMV over thread tile T, CTA size C, slice count

@@ -386,6 +386,48 @@ yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host
   return YASPMV_OK;
 }
 
+yaspmv_status yaspmv_spmv_host_async(yaspmv_matrix A, const void* x_host, void* y_host, void* stream) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle: no CPU fallback");
+  const size_t xb = (size_t)A->can.n * A->vsize, yb = (size_t)A->can.m * A->vsize;
+  CUDA_TRY(cudaSetDevice(A->device));
+  if (!A->s_in) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&A->s_in, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&A->s_out, cudaStreamNonBlocking));
+    for (auto& s : A->hslot) {
+      CUDA_TRY(cudaMalloc(&s.x, std::max<size_t>(xb, 16)));
+      CUDA_TRY(cudaMalloc(&s.y, std::max<size_t>(yb, 16)));
+      CUDA_TRY(cudaEventCreateWithFlags(&s.in, cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&s.comp, cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
+      CUDA_TRY(cudaEventRecord(s.done, A->s_out));
+    }
+  }
+  auto& s = A->hslot[A->next_slot];
+  A->next_slot ^= 1;
+  cudaStream_t cs = (cudaStream_t)stream;
+  CUDA_TRY(cudaStreamWaitEvent(A->s_in, s.done, 0));  // the slot's previous copy-out is done
+  if (xb) CUDA_TRY(cudaMemcpyAsync(s.x, x_host, xb, cudaMemcpyHostToDevice, A->s_in));
+  CUDA_TRY(cudaEventRecord(s.in, A->s_in));
+  CUDA_TRY(cudaStreamWaitEvent(cs, s.in, 0));
+  yaspmv_status st = run_spmv(A, s.x, s.y, stream);
+  if (st != YASPMV_OK) return st;
+  CUDA_TRY(cudaEventRecord(s.comp, cs));
+  CUDA_TRY(cudaStreamWaitEvent(A->s_out, s.comp, 0));
+  if (yb) CUDA_TRY(cudaMemcpyAsync(y_host, s.y, yb, cudaMemcpyDeviceToHost, A->s_out));
+  CUDA_TRY(cudaEventRecord(s.done, A->s_out));
+  return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_host_sync(yaspmv_matrix A) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->s_out) {
+    CUDA_TRY(cudaSetDevice(A->device));
+    CUDA_TRY(cudaStreamSynchronize(A->s_out));
+  }
+  return YASPMV_OK;
+}
+
 int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
   if (!A || A->can.m == 0) return 0;
   if (A->can.ntiles == 0) return 0;  // memset only

@@ -44,6 +44,14 @@ struct yaspmv_matrix_s {
   int64_t grid = 1;  // persistent CTAs per launch (fixed per encoding: ticket period)
   void* xs = nullptr;  // scratch for spmv_host
   void* ys = nullptr;
+  // spmv_host_async: two buffer slots, two copy streams, chaining events
+  struct HostSlot {
+    void* x = nullptr;
+    void* y = nullptr;
+    cudaEvent_t in = nullptr, comp = nullptr, done = nullptr;
+  } hslot[2];
+  cudaStream_t s_in = nullptr, s_out = nullptr;
+  int next_slot = 0;
   int64_t n_escapes = 0;
   double build_s = 0, tune_s = 0;
   int tune_candidates = 0;
@@ -55,6 +63,16 @@ struct yaspmv_matrix_s {
       d.free_all();
       if (xs) cudaFree(xs);
       if (ys) cudaFree(ys);
+      if (s_out) cudaStreamSynchronize(s_out);
+      for (auto& s : hslot) {
+        if (s.x) cudaFree(s.x);
+        if (s.y) cudaFree(s.y);
+        if (s.in) cudaEventDestroy(s.in);
+        if (s.comp) cudaEventDestroy(s.comp);
+        if (s.done) cudaEventDestroy(s.done);
+      }
+      if (s_in) cudaStreamDestroy(s_in);
+      if (s_out) cudaStreamDestroy(s_out);
       cudaSetDevice(cur);
     }
   }

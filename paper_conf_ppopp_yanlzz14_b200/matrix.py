@@ -114,6 +114,14 @@ class Matrix:
         check(lib.yaspmv_spmv_host(self._h, _ptr(x), _ptr(y), _stream(stream) if stream != 0 else 0))
         return y
 
+    def spmv_host_async(self, x: np.ndarray, y: np.ndarray, stream=None) -> None:
+        """Queue y := A·x with host arrays (pinned for overlap); call host_sync() before
+        reading y or reusing x."""
+        check(lib.yaspmv_spmv_host_async(self._h, _ptr(x), _ptr(y), _stream(stream) if stream != 0 else 0))
+
+    def host_sync(self) -> None:
+        check(lib.yaspmv_host_sync(self._h))
+
     def tune(self, stream=None) -> dict:
         p = _lib.Params()
         check(lib.yaspmv_tune(self._h, _stream(stream), ctypes.byref(p)))

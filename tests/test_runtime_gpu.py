@@ -1,0 +1,93 @@
+"""Runtime properties of the CUDA path: CUDA-graph replay (the per-launch epoch and ticket
+live on the device, so replays stay correct), the pipelined host API, and a
+compute-sanitizer memcheck / synccheck run of the kernels."""
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import ref
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def test_cuda_graph_replay():
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    csr = synth.webbase_like(m=200_000, integer=True)
+    A = Matrix.from_synth(csr, device=0, T=8, C=128, S=2)
+    xs = [synth.make_x(csr.n, np.float32, "int2", s) for s in range(3)]
+    x = torch.from_numpy(xs[0]).cuda()
+    y = torch.empty(csr.m, dtype=torch.float32, device="cuda")
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        A.spmv(x, y)  # warm-up outside capture
+    torch.cuda.current_stream().wait_stream(s)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        A.spmv(x, y)
+        A.spmv(x, y)
+    for k in range(3):
+        x.copy_(torch.from_numpy(xs[k]))
+        g.replay()
+        torch.cuda.synchronize()
+        ye, _ = ref.spmv(csr.row_ptr, csr.col, csr.val, xs[k])
+        assert np.array_equal(y.cpu().numpy().astype(np.float64), ye)
+    A.free()
+
+
+def test_host_async_pipeline():
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    csr = synth.fem_like("cantilever", integer=True)
+    A = Matrix.from_synth(csr, device=0, h=4, w=4, T=4, C=128)
+    xs = [torch.from_numpy(synth.make_x(csr.n, np.float32, "int2", s)).pin_memory() for s in range(4)]
+    ys = [torch.empty(csr.m, dtype=torch.float32).pin_memory() for _ in range(4)]
+    for k in range(4):
+        A.spmv_host_async(xs[k].numpy(), ys[k].numpy())
+    A.host_sync()
+    for k in range(4):
+        ye, _ = ref.spmv(csr.row_ptr, csr.col, csr.val, xs[k].numpy())
+        assert np.array_equal(ys[k].numpy().astype(np.float64), ye)
+    A.free()
+
+
+SANITIZE = r"""
+import numpy as np, torch, sys
+sys.path.insert(0, %r)
+import synth
+from paper_conf_ppopp_yanlzz14_b200 import Matrix
+csr = synth.webbase_like(m=20000)
+x = torch.from_numpy(synth.make_x(csr.n, np.float32, "unit", 0)).cuda()
+for p in (dict(T=4, C=64), dict(T=16, C=256, S=3, empty_mode=2), dict(T=8, C=128, col_mode=3)):
+    A = Matrix.from_synth(csr, device=0, **p)
+    A.spmv(x); torch.cuda.synchronize(); A.free()
+c = synth.fem_like("cantilever")
+A = Matrix.from_synth(c, device=0, h=4, w=4, T=4, C=128)
+A.spmv(torch.from_numpy(synth.make_x(c.n, np.float32, "uniform", 0)).cuda()); torch.cuda.synchronize()
+print("SANITIZE-DONE")
+""" % ROOT
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "synccheck"])
+def test_compute_sanitizer(tool, tmp_path):
+    exe = "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(exe):
+        pytest.skip("compute-sanitizer not available")
+    script = tmp_path / "san.py"
+    script.write_text(SANITIZE)
+    r = subprocess.run([exe, "--tool", tool, "--error-exitcode", "9", "--kernel-name", "kns=yaspmv",
+                        sys.executable, str(script)], capture_output=True, text=True, timeout=900)
+    assert "SANITIZE-DONE" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
+    assert r.returncode == 0, r.stdout[-3000:]
+    assert "ERROR SUMMARY: 0 errors" in r.stdout
