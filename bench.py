@@ -265,18 +265,20 @@ def main():
     if world > 1:
         dist.barrier()
     e0.record(stream)
+    L_ = L
     for k in range(args.steps):
-        # SpMV launches recorded separately: the dominant kernel's live duration
+        # the fused step: SpMV kernel with the 1/||z_{k-1}|| scaling and ||z_k||^2 partials in
+        # its epilogue (+ 2 tiny reduction kernels); events bracket it on the launching stream
         ev[k][0].record(stream)
-        ops.spmv(pit.x, pit.y[: L.m_local])
+        ops.power_step(pit.x, pit.y[: L_.m_local], None if pit.first else pit.norm_prev, pit.norm2)
         ev[k][1].record(stream)
-        ops.nrm2sq(pit.y[: L.m_local], pit.norm2)
+        pit.first = False
         if world > 1:
             dist.all_reduce(pit.norm2)
-            ops.scale(pit.y[: L.m_local], pit.y[: L.m_local], pit.norm2)
             dist.all_gather_into_tensor(pit.x, pit.y)
         else:
-            ops.scale(pit.y[: L.m_local], pit.x[: L.m_local], pit.norm2)
+            pit.x, pit.y = pit.y, pit.x
+        pit.norm_prev, pit.norm2 = pit.norm2, pit.norm_prev
     e1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -302,7 +304,7 @@ def main():
     # every step copies x host->device and y device->host; yaspmv_spmv_host_async overlaps
     # the copies of consecutive steps with the SpMV (two buffer slots, two copy streams)
     xh = torch.empty(L.n_padded, dtype=tdt).pin_memory()
-    xh.copy_(pit.x.cpu())
+    xh.copy_(pit.current_x().cpu())
     yh = torch.empty(L.m_local, dtype=tdt).pin_memory()
     A.spmv_host_async(xh.numpy(), yh.numpy(), stream=stream.cuda_stream)
     A.host_sync()
@@ -341,21 +343,22 @@ def main():
                        "params": info["params"], "parallelism": f"row-partition x{world}, NCCL all-gather of x",
                        "l2": "inputs larger than L2 (matrix 8.5 GB vs 126 MB L2), no flush" if args.config == "c5"
                        else "L2-resident workload; back-to-back steps (warm L2)",
-                       "step": "y=A x (fused BCCOO SpMV) + ||y||^2 + scale" + (" + allreduce + allgather" if world > 1 else "")},
+                       "step": "z_k = A z_{k-1}/||z_{k-1}|| and ||z_k||^2 in one fused BCCOO SpMV launch (+2 tiny sums)"
+                               + (" + NCCL allreduce(1 fp64) + allgather(z)" if world > 1 else "")},
             "spmv_ms": spmv_ms, "spmv_ms_max_over_ranks": spmv_ms_max,
             "spmv_gflops": 2.0 * info["nnz"] / (spmv_ms * 1e-3) / 1e9,
             "hbm_gbs_alg": achieved, "pct_of_8TBs": achieved / 8000.0 * 100.0,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "spmv_bccoo_kernel" + (" + combine" if info["params"]["slices"] > 1 else ""),
+                         "kernel": "spmv_bccoo_kernel" + (" + combine" if info["params"]["slices"] > 1 else "")
+                                   + " (+ 2 tiny y^2-partial reductions of the fused step)",
                          "alg_bytes_per_launch": info["alg_bytes"]},
-            "gpu_launches": (A.launches_per_spmv() + 3) * args.steps,
+            "gpu_launches": A.launches_per_power_step() * args.steps,
             "clocks": clocks, "e2e": e2e,
             "build": {"generate_s": t_gen, "build_s": t_build, "encode_upload_s": info["build_seconds"]},
         }
         if world == 1 and not args.no_cpu_baseline:
-            x_np = pit.x[: L.m_local].float().cpu().numpy().astype(dtype_np) if args.config == "c5" \
-                else pit.x.cpu().numpy()
+            x_np = pit.current_x()[: L.m_local].cpu().numpy().astype(dtype_np)
             if args.config == "c5":
                 line["cpu_baseline"] = cpu_baseline(csr, x_np)
             else:

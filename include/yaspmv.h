@@ -127,6 +127,17 @@ void yaspmv_free(yaspmv_matrix A);
  * combine. */
 yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream);
 
+/* yaspmv_spmv_power: one step of the power iteration fused into the SpMV (not in the
+ * paper; BASELINE.json's iterated SpMV):  y := (A·x) / sqrt(in_norm2[0])  (no scaling if
+ * in_norm2 is NULL) and, if out_norm2 is not NULL, out_norm2[0] := sum_i y[i]^2 (fp64,
+ * deterministic fixed-tree reduction).  in_norm2 / out_norm2 are DEVICE doubles.  With
+ * z_k = A x_k, calling it on (z_{k-1}, ||z_{k-1}||^2) yields z_k and ||z_k||^2 without a
+ * separate normalisation pass.  Launches: the SpMV (+ the BCCOO+ combine, which then does
+ * the scaling and the partial sums) + two small reduction kernels. */
+yaspmv_status yaspmv_spmv_power(yaspmv_matrix A, const void* x, void* y, const double* in_norm2, double* out_norm2,
+                                void* stream);
+int32_t yaspmv_launches_per_power_step(yaspmv_matrix A);
+
 /* yaspmv_spmv_host: y := A·x with HOST x / y: copies x host->device into handle-owned
  * scratch, runs yaspmv_spmv, copies y device->host, and synchronizes `stream` before
  * returning.  Pinned host memory gives full PCIe/NVLink-C2C bandwidth. */

@@ -25,7 +25,8 @@ ARR = {"flags": 0, "col": 1, "col_delta": 2, "val0": 3, "val1": 4, "val2": 5, "v
 EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv", "yaspmv_spmv_host",
             "yaspmv_tune", "yaspmv_reencode", "yaspmv_get_info", "yaspmv_export", "yaspmv_export_device",
             "yaspmv_nrm2sq", "yaspmv_nrm2sq_scratch_bytes", "yaspmv_scale", "yaspmv_last_error",
-            "yaspmv_version", "yaspmv_launches_per_spmv", "yaspmv_spmv_host_async", "yaspmv_host_sync"]
+            "yaspmv_version", "yaspmv_launches_per_spmv", "yaspmv_spmv_host_async", "yaspmv_host_sync",
+            "yaspmv_spmv_power", "yaspmv_launches_per_power_step"]
 
 
 class Params(ctypes.Structure):
@@ -90,6 +91,8 @@ def _load():
         "yaspmv_launches_per_spmv": ([H], i32),
         "yaspmv_spmv_host_async": ([H, vp, vp, vp], ctypes.c_int),
         "yaspmv_host_sync": ([H], ctypes.c_int),
+        "yaspmv_spmv_power": ([H, vp, vp, vp, vp, vp], ctypes.c_int),
+        "yaspmv_launches_per_power_step": ([H], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

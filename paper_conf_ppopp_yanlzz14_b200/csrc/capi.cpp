@@ -255,13 +255,31 @@ int64_t alg_bytes(const yaspmv_matrix A) {
   return b;
 }
 
-yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
+yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2 = nullptr,
+                       double* out_norm2 = nullptr) {
   const Canonical& c = A->can;
   const Params& p = c.p;
-  if (c.m == 0) return YASPMV_OK;
-  if (c.ntiles == 0) {
-    CUDA_TRY(cudaMemsetAsync(y, 0, (size_t)c.m * A->vsize, (cudaStream_t)stream));
+  cudaStream_t cs = (cudaStream_t)stream;
+  if (c.m == 0) {
+    if (out_norm2) CUDA_TRY(cudaMemsetAsync(out_norm2, 0, sizeof(double), cs));
     return YASPMV_OK;
+  }
+  if (c.ntiles == 0) {
+    CUDA_TRY(cudaMemsetAsync(y, 0, (size_t)c.m * A->vsize, cs));
+    if (out_norm2) CUDA_TRY(cudaMemsetAsync(out_norm2, 0, sizeof(double), cs));
+    return YASPMV_OK;
+  }
+  const int nw1 = p.C / 32 + 1;
+  const int64_t npart = p.S == 1 ? c.ntiles * nw1 : combine_blocks(c.m);
+  if (out_norm2 && A->npart < npart) {  // partial sums of y^2 + the reduction scratch
+    if (A->d_part) cudaFree(A->d_part);
+    if (A->d_scratch) cudaFree(A->d_scratch);
+    A->d_part = nullptr;
+    A->d_scratch = nullptr;
+    A->npart = 0;
+    CUDA_TRY(cudaMalloc((void**)&A->d_part, npart * sizeof(double)));
+    CUDA_TRY(cudaMalloc((void**)&A->d_scratch, nrm2sq_blocks(npart) * sizeof(double)));
+    A->npart = npart;
   }
   KArgs a;
   for (int r = 0; r < 4; ++r) a.val[r] = A->d.val[r];
@@ -281,10 +299,18 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
   a.ticket = A->d.ticket;
   a.status = A->d.status;
   a.carry = A->d.carry;
+  a.epi = 0;
+  a.in_norm2 = in_norm2;
+  a.part = A->d_part;
+  if (p.S == 1) a.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
   A->kern->launch(a, p.C, A->grid, stream);
   CUDA_TRY(cudaGetLastError());
   if (p.S > 1) {
-    launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream);
+    launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream, in_norm2, out_norm2 ? A->d_part : nullptr);
+    CUDA_TRY(cudaGetLastError());
+  }
+  if (out_norm2) {
+    launch_sum_f64(A->d_part, npart, out_norm2, A->d_scratch, stream);
     CUDA_TRY(cudaGetLastError());
   }
   return YASPMV_OK;
@@ -370,6 +396,21 @@ yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream)
   return run_spmv(A, x, y, stream);
 }
 
+yaspmv_status yaspmv_spmv_power(yaspmv_matrix A, const void* x, void* y, const double* in_norm2, double* out_norm2,
+                                void* stream) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle (built with device = -1): no CPU fallback");
+  if (A->can.m > 0 && !y) return fail(YASPMV_EINVAL, "y is NULL");
+  if (A->can.n > 0 && !x) return fail(YASPMV_EINVAL, "x is NULL");
+  const int64_t xb = A->can.n * A->vsize, yb = A->can.m * A->vsize;
+  const char* xc = static_cast<const char*>(x);
+  const char* yc = static_cast<const char*>(y);
+  if (xb > 0 && yb > 0 && xc < yc + yb && yc < xc + xb) return fail(YASPMV_EINVAL, "x and y overlap");
+  if (((uintptr_t)x) % ((uintptr_t)A->can.p.w * A->vsize) != 0)
+    return fail(YASPMV_EINVAL, "x must be aligned to w * sizeof(value) bytes");
+  return run_spmv(A, x, y, stream, in_norm2, out_norm2);
+}
+
 yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host, void* stream) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle: no CPU fallback");
@@ -432,6 +473,11 @@ int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
   if (!A || A->can.m == 0) return 0;
   if (A->can.ntiles == 0) return 0;  // memset only
   return A->can.p.S > 1 ? 2 : 1;
+}
+
+int32_t yaspmv_launches_per_power_step(yaspmv_matrix A) {
+  if (!A || A->can.m == 0 || A->can.ntiles == 0) return 0;
+  return yaspmv_launches_per_spmv(A) + 2;  // + the two-level sum of the y^2 partials
 }
 
 yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {

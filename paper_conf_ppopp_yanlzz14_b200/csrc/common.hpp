@@ -97,6 +97,11 @@ struct KArgs {
   unsigned long long* ticket;
   unsigned long long* status;
   double* carry;           // ntiles * h
+  // power-iteration epilogue (yaspmv_spmv_power): bit 0 scale y by 1/sqrt(*in_norm2),
+  // bit 1 write per-warp partials of sum y^2 to part[tile*(C/32+1) + warp] (+ carried seg)
+  int epi;
+  const double* in_norm2;
+  double* part;
 };
 
 typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
@@ -111,7 +116,10 @@ struct KernelEntry {
 const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm);
 const std::vector<KernelEntry>& all_kernels();
 
-void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream);
+void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream,
+                    const double* in_norm2 = nullptr, double* part = nullptr);
+int64_t combine_blocks(int64_t m);
+void launch_sum_f64(const double* v, int64_t n, double* out, double* partials, void* stream);
 void launch_nrm2sq(const void* v, int64_t n, int dtype, double* out, double* partials, void* stream);
 int64_t nrm2sq_blocks(int64_t n);
 void launch_scale(const void* src, void* dst, int64_t n, int dtype, const double* norm2, void* stream);

@@ -52,6 +52,9 @@ struct yaspmv_matrix_s {
   } hslot[2];
   cudaStream_t s_in = nullptr, s_out = nullptr;
   int next_slot = 0;
+  double* d_part = nullptr;     // power-iteration epilogue: partials of sum y^2
+  double* d_scratch = nullptr;  // two-level reduction scratch
+  int64_t npart = 0;
   int64_t n_escapes = 0;
   double build_s = 0, tune_s = 0;
   int tune_candidates = 0;
@@ -72,6 +75,8 @@ struct yaspmv_matrix_s {
         if (s.done) cudaEventDestroy(s.done);
       }
       if (s_in) cudaStreamDestroy(s_in);
+      if (d_part) cudaFree(d_part);
+      if (d_scratch) cudaFree(d_scratch);
       if (s_out) cudaStreamDestroy(s_out);
       cudaSetDevice(cur);
     }

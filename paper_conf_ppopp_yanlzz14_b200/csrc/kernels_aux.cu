@@ -11,13 +11,25 @@ namespace yaspmv {
 // ---------------------------------------------------------------- BCCOO+ combine
 // y[i] = sum_{s=0..S-1} tmp[s*stride + i], ascending s (Fig. 5; Q11), fp64
 // accumulation then one rounding.  Vectorised 4 elements per thread when aligned.
+__device__ __forceinline__ double block_sum256(double v);
+
+// optional power-iteration epilogue: y scaled by 1/sqrt(*in_norm2), block partials of y^2
 template <typename VT>
-__global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, int64_t m, int64_t stride, int S) {
+__global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, int64_t m, int64_t stride, int S,
+                               const double* __restrict__ in_norm2, double* __restrict__ part) {
   const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+  const double inv = in_norm2 ? 1.0 / sqrt(in_norm2[0]) : 1.0;
+  double ss = 0.0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += nthreads) {
     double s = (double)__ldcs(tmp + i);
     for (int q = 1; q < S; ++q) s += (double)__ldcs(tmp + (int64_t)q * stride + i);
-    y[i] = (VT)s;
+    const VT o = in_norm2 ? (VT)((VT)s * inv) : (VT)s;
+    y[i] = o;
+    ss += (double)o * (double)o;
+  }
+  if (part) {
+    ss = block_sum256(ss);
+    if (threadIdx.x == 0) part[blockIdx.x] = ss;
   }
 }
 
@@ -32,15 +44,23 @@ static int num_sms() {
   return sms;
 }
 
-void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream) {
-  if (m <= 0) return;
+int64_t combine_blocks(int64_t m) {
   int64_t blocks = (m + 255) / 256;
-  const int64_t cap = (int64_t)num_sms() * 8;
+  const int64_t cap = (int64_t)num_sms() * 16;
   if (blocks > cap) blocks = cap;
+  return blocks < 1 ? 1 : blocks;
+}
+
+void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream,
+                    const double* in_norm2, double* part) {
+  if (m <= 0) return;
+  const int64_t blocks = combine_blocks(m);
   if (dtype == 0)
-    combine_kernel<float><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const float*)tmp, (float*)y, m, stride, S);
+    combine_kernel<float><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const float*)tmp, (float*)y, m,
+                                                                             stride, S, in_norm2, part);
   else
-    combine_kernel<double><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const double*)tmp, (double*)y, m, stride, S);
+    combine_kernel<double><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const double*)tmp, (double*)y, m,
+                                                                               stride, S, in_norm2, part);
 }
 
 // ---------------------------------------------------------------- ||v||^2
@@ -78,6 +98,16 @@ __global__ void nrm2sq_partial(const VT* __restrict__ v, int64_t n, double* __re
   if (threadIdx.x == 0) partials[blockIdx.x] = s;
 }
 
+__device__ __forceinline__ double block_sum256(double v) { return block_sum(v); }
+
+__global__ void sum_f64_partial(const double* __restrict__ v, int64_t n, double* __restrict__ partials) {
+  double s = 0.0;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) s += v[i];
+  s = block_sum(s);
+  if (threadIdx.x == 0) partials[blockIdx.x] = s;
+}
+
 __global__ void nrm2sq_final(const double* __restrict__ partials, int nb, double* __restrict__ out) {
   double s = 0.0;
   for (int i = threadIdx.x; i < nb; i += blockDim.x) s += partials[i];
@@ -90,6 +120,14 @@ void launch_nrm2sq(const void* v, int64_t n, int dtype, double* out, double* par
   cudaStream_t st = (cudaStream_t)stream;
   if (dtype == 0) nrm2sq_partial<float><<<(unsigned)nb, NRM_THREADS, 0, st>>>((const float*)v, n, partials);
   else nrm2sq_partial<double><<<(unsigned)nb, NRM_THREADS, 0, st>>>((const double*)v, n, partials);
+  nrm2sq_final<<<1, NRM_THREADS, 0, st>>>(partials, (int)nb, out);
+}
+
+// deterministic sum of n doubles (fixed grid for a given n): out[0] = sum v
+void launch_sum_f64(const double* v, int64_t n, double* out, double* partials, void* stream) {
+  const int64_t nb = nrm2sq_blocks(n);
+  cudaStream_t st = (cudaStream_t)stream;
+  sum_f64_partial<<<(unsigned)nb, NRM_THREADS, 0, st>>>(v, n, partials);
   nrm2sq_final<<<1, NRM_THREADS, 0, st>>>(partials, (int)nb, out);
 }
 

@@ -160,6 +160,7 @@ template <typename VT, int H>
 struct ScanShared {
   long long tile;
   unsigned long long epoch;
+  double inv;  // power-iteration epilogue scale 1/sqrt(*in_norm2), computed once per CTA
   VT wv[16][H];
   int wf[16];
   int wn[16];
@@ -167,7 +168,7 @@ struct ScanShared {
 
 // The work of one workgroup-level tile (T*C consecutive blocks): steps 1-3
 // of P:226 plus the cross-tile carry.
-template <typename VT, int H, int W, int T, int CM>
+template <typename VT, int H, int W, int T, int CM, bool EPI>
 __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, const unsigned long long epoch,
                                           ScanShared<VT, H>& sh) {
   using TR = KTraits<VT, H, W, T, CM>;
@@ -319,39 +320,87 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
   // ---- step 2c/3b: combine and write back -----------------------------
   const bool dependent = hs && !Fex && tile > 0;  // the tile's first stop needs the carry
   const int64_t seg0 = (int64_t)__ldg(a.cta_seg0 + tile) + Nex;  // first-result entry
+  // optional power-iteration epilogue: y scaled by 1/sqrt(in_norm2), sum y^2 partials
+  const double inv = EPI ? sh.inv : 1.0;
+  const VT invv = (VT)inv;
+  VT ssv = VT(0);
   VT dep[H];
   int64_t dep_row = 0;
   if (hs) {
+    // Strategy 1 combine: walk the intermediate sums; the first stop adds the
+    // scanned last partial sums of earlier threads (Vex), later stops are complete.  The
+    // tile's very first segment (dependent) is handed to the look-back below.
     VT run[H];
 #pragma unroll
-    for (int r = 0; r < H; ++r) run[r] = Vex[r];  // the segment's part in earlier threads
-    int j = 0;
+    for (int r = 0; r < H; ++r) run[r] = Vex[r];
+    bool first = dependent;
+    if (a.seg_row == nullptr) {  // segment k is stacked row k: rows are consecutive
+      int64_t row = seg0;
 #pragma unroll
-    for (int b = 0; b < T; ++b) {
+      for (int b = 0; b < T; ++b) {
 #pragma unroll
-      for (int r = 0; r < H; ++r) run[r] = run[r] + pr[b][r];
-      if ((stops >> b) & 1u) {
-        const int64_t seg = seg0 + j;
-        const int64_t sr = a.seg_row ? (int64_t)__ldg(a.seg_row + seg) : seg;
-        if (j == 0 && dependent) {
+        for (int r = 0; r < H; ++r) run[r] = run[r] + pr[b][r];
+        if ((stops >> b) & 1u) {
+          if (first) {
 #pragma unroll
-          for (int r = 0; r < H; ++r) dep[r] = run[r];
-          dep_row = sr;
-        } else {
+            for (int r = 0; r < H; ++r) dep[r] = run[r];
+            dep_row = row;
+          } else {
+            VT* op = out + row * H;
 #pragma unroll
-          for (int r = 0; r < H; ++r)
-            if (sr * H + r < a.out_limit) out[sr * H + r] = run[r];
+            for (int r = 0; r < H; ++r)
+              if (H == 1 || row * H + r < a.out_limit) {
+                const VT o = EPI ? run[r] * invv : run[r];
+                op[r] = o;
+                if constexpr (EPI) ssv = fma(o, o, ssv);
+              }
+          }
+          first = false;
+          ++row;
+#pragma unroll
+          for (int r = 0; r < H; ++r) run[r] = VT(0);
         }
-        ++j;
+      }
+    } else {  // seg_row map (empty_mode MAP, Q1)
+      int64_t seg = seg0;
 #pragma unroll
-        for (int r = 0; r < H; ++r) run[r] = VT(0);
+      for (int b = 0; b < T; ++b) {
+#pragma unroll
+        for (int r = 0; r < H; ++r) run[r] = run[r] + pr[b][r];
+        if ((stops >> b) & 1u) {
+          const int64_t sr = (int64_t)__ldg(a.seg_row + seg);
+          if (first) {
+#pragma unroll
+            for (int r = 0; r < H; ++r) dep[r] = run[r];
+            dep_row = sr;
+          } else {
+#pragma unroll
+            for (int r = 0; r < H; ++r)
+              if (sr * H + r < a.out_limit) {
+                const VT o = EPI ? run[r] * invv : run[r];
+                out[sr * H + r] = o;
+                if constexpr (EPI) ssv = fma(o, o, ssv);
+              }
+          }
+          first = false;
+          ++seg;
+#pragma unroll
+          for (int r = 0; r < H; ++r) run[r] = VT(0);
+        }
       }
     }
   }
+  double ss = (double)ssv;
 
   // ---- step 3c: look back for the carry-in (decoupled look-back) --------
   // by the warp holding the tile's first row stop; a window of 32 predecessors per
   // round, polled with relaxed loads (no L1 invalidation: x stays cached in L1)
+  if (EPI && (a.epi & 2)) {  // per-warp partial of sum y^2, fixed tree (deterministic)
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+    if (lane == 0) a.part[tile * (NW + 1) + wid] = ss;
+    if (t == 0 && !(Fall && tile > 0)) a.part[tile * (NW + 1) + NW] = 0.0;  // no carried segment
+  }
   const unsigned dep_ballot = __ballot_sync(0xffffffffu, dependent);
   if (dep_ballot == 0) return;
   const int dep_lane = __ffs(dep_ballot) - 1;
@@ -382,9 +431,15 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
     jw -= 32;
   }
   if (lane == dep_lane) {
+    double ds = 0.0;
 #pragma unroll
     for (int r = 0; r < H; ++r)
-      if (dep_row * H + r < a.out_limit) out[dep_row * H + r] = (VT)((double)dep[r] + carry[r]);
+      if (dep_row * H + r < a.out_limit) {
+        const VT o = (VT)(((double)dep[r] + carry[r]) * inv);
+        out[dep_row * H + r] = o;
+        ds += (double)o * (double)o;
+      }
+    if (EPI && (a.epi & 2)) a.part[tile * (NW + 1) + NW] = ds;
   }
 }
 
@@ -392,7 +447,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
 #ifndef YASPMV_MINB
 #define YASPMV_MINB 1
 #endif
-template <typename VT, int H, int W, int T, int CM>
+template <typename VT, int H, int W, int T, int CM, bool EPI>
 __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) spmv_bccoo_kernel(const KArgs a) {
   __shared__ ScanShared<VT, H> sh;
   if (threadIdx.x == 0) {
@@ -400,21 +455,24 @@ __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) s
     const unsigned long long q = tk / (unsigned long long)a.period;
     sh.tile = (long long)(tk - q * (unsigned long long)a.period);
     sh.epoch = q + 1ull;  // launches so far: tags this launch's status words (Q9)
+    if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   }
   __syncthreads();
-  tile_body<VT, H, W, T, CM>(a, sh.tile, sh.epoch, sh);
+  tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, sh.epoch, sh);
 }
 
 template <typename VT, int H, int W, int T, int CM>
 void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
   using TR = KTraits<VT, H, W, T, CM>;
-  spmv_bccoo_kernel<VT, H, W, T, CM><<<(unsigned)grid, C, TR::smem_bytes(C), (cudaStream_t)stream>>>(a);
+  if (a.epi) spmv_bccoo_kernel<VT, H, W, T, CM, true><<<(unsigned)grid, C, TR::smem_bytes(C), (cudaStream_t)stream>>>(a);
+  else spmv_bccoo_kernel<VT, H, W, T, CM, false><<<(unsigned)grid, C, TR::smem_bytes(C), (cudaStream_t)stream>>>(a);
 }
 
 template <typename VT, int H, int W, int T, int CM>
 int attr_spmv(int C, int* regs, int* max_threads, int* blocks_per_sm) {
   using TR = KTraits<VT, H, W, T, CM>;
-  auto k = spmv_bccoo_kernel<VT, H, W, T, CM>;
+  auto k = spmv_bccoo_kernel<VT, H, W, T, CM, false>;
+  auto k2 = spmv_bccoo_kernel<VT, H, W, T, CM, true>;
   cudaFuncAttributes fa;
   cudaError_t e = cudaFuncGetAttributes(&fa, k);
   if (e != cudaSuccess) return (int)e;
@@ -430,6 +488,8 @@ int attr_spmv(int C, int* regs, int* max_threads, int* blocks_per_sm) {
     if (e != cudaSuccess) return (int)e;
     // x gathers are the L1 traffic: give L1 the whole unified carve-out
     e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
+    if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(k2, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
     if (e != cudaSuccess) return (int)e;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k, C, TR::smem_bytes(C));
     if (e != cudaSuccess) return (int)e;

@@ -81,7 +81,9 @@ def make_layout(row_ptr: np.ndarray, rank: int, world: int, h: int = 1) -> Layou
 
 
 class GpuOps:
-    """Local steps on the GPU: the fused SpMV kernel(s) + ||y||^2 + scale (libyaspmv)."""
+    """Local steps on the GPU (libyaspmv): the fused power step — the BCCOO SpMV kernel
+    with its epilogue scaling y by 1/||z_prev|| and producing the partials of ||y||^2 —
+    plus the plain SpMV / norm / scale kernels for the unfused path."""
 
     def __init__(self, A, n_local_rows: int, device):
         import torch
@@ -90,6 +92,9 @@ class GpuOps:
         self.A = A
         self.scratch = torch.zeros(nrm2sq_scratch_bytes(max(n_local_rows, 1)) // 8 + 1, dtype=torch.float64,
                                    device=device)
+
+    def power_step(self, v, z, in_norm2, out_norm2):
+        self.A.spmv_power(v, z, in_norm2, out_norm2)
 
     def spmv(self, x, y):
         self.A.spmv(x, y)
@@ -103,20 +108,29 @@ class GpuOps:
         scale(src, dst, norm2)
 
     def launches_per_step(self) -> int:
-        return self.A.launches_per_spmv() + 3  # + nrm2sq (2) + scale (1)
+        return self.A.launches_per_power_step()
 
 
 class PowerIteration:
-    """x_{k+1} = A x_k / ||A x_k|| with A row-partitioned over the process group."""
+    """x_{k+1} = A x_k / ||A x_k|| with A row-partitioned over the process group.
+
+    Fused form (ops with ``power_step``): the iterate is kept unnormalised, z_k = A x_k,
+    and x_k = z_{k-1} / ||z_{k-1}|| is never materialised — each step is one SpMV launch
+    whose epilogue applies 1/||z_{k-1}|| and produces ||z_k||^2 partials, then one scalar
+    all-reduce and the all-gather of z_k's row blocks (N > 1).  Unfused form (ops with
+    spmv / nrm2sq / scale): normalise explicitly after every SpMV."""
 
     def __init__(self, layout: Layout, ops, dtype, device, group=None):
         import torch
         self.L = layout
         self.ops = ops
         self.group = group
-        self.x = torch.zeros(layout.n_padded, dtype=dtype, device=device)
-        self.y = torch.zeros(layout.m_max, dtype=dtype, device=device)   # padded local block
+        self.fused = hasattr(ops, "power_step")
+        self.x = torch.zeros(layout.n_padded, dtype=dtype, device=device)      # replicated vector
+        self.y = torch.zeros(layout.m_max, dtype=dtype, device=device)         # padded local block
         self.norm2 = torch.zeros(1, dtype=torch.float64, device=device)
+        self.norm_prev = torch.ones(1, dtype=torch.float64, device=device)     # ||z_{k-1}||^2 (1: x_0)
+        self.first = True
         n_true = int(layout.bounds[-1])
         for r in range(layout.world):  # x_0 = 1/sqrt(N) on the real entries
             a = r * layout.m_max
@@ -126,12 +140,29 @@ class PowerIteration:
         import torch.distributed as dist
         L = self.L
         y_loc = self.y[: L.m_local]
-        self.ops.spmv(self.x, y_loc)                    # y_r = A_r x   (fused SpMV kernel)
+        if self.fused:
+            # z_k = (A z_{k-1}) / ||z_{k-1}||  and  ||z_k||^2  (one SpMV launch + 2 tiny sums)
+            self.ops.power_step(self.x, y_loc, None if self.first else self.norm_prev, self.norm2)
+            self.first = False
+            if L.world > 1:
+                dist.all_reduce(self.norm2, group=self.group)                  # 1 fp64 over NVLink
+                dist.all_gather_into_tensor(self.x, self.y, group=self.group)  # replicate z_k
+            else:
+                self.x, self.y = self.y, self.x                                  # z_k is the next input
+            self.norm_prev, self.norm2 = self.norm2, self.norm_prev
+            return self.x
+        self.ops.spmv(self.x, y_loc)                    # y_r = A_r x
         self.ops.nrm2sq(y_loc, self.norm2)              # ||y_r||^2
         if L.world > 1:
-            dist.all_reduce(self.norm2, group=self.group)          # 1 fp64 over NVLink
+            dist.all_reduce(self.norm2, group=self.group)
             self.ops.scale(y_loc, y_loc, self.norm2)
-            dist.all_gather_into_tensor(self.x, self.y, group=self.group)  # replicate x
+            dist.all_gather_into_tensor(self.x, self.y, group=self.group)
         else:
             self.ops.scale(y_loc, self.x[: L.m_local], self.norm2)
+        return self.x
+
+    def current_x(self):
+        """The normalised iterate x_k (materialised; for checks)."""
+        if self.fused and not self.first:
+            return self.x / self.norm_prev.sqrt().to(self.x.dtype)
         return self.x

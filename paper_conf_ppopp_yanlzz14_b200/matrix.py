@@ -106,6 +106,15 @@ class Matrix:
         check(lib.yaspmv_spmv(self._h, _ptr(x), _ptr(y), _stream(stream)))
         return y
 
+    def spmv_power(self, x, y, in_norm2=None, out_norm2=None, stream=None):
+        """y := (A·x)/sqrt(in_norm2[0]) and out_norm2[0] := sum y^2 (device tensors; either
+        norm may be None) — one fused power-iteration step."""
+        check(lib.yaspmv_spmv_power(self._h, _ptr(x), _ptr(y), _ptr(in_norm2), _ptr(out_norm2), _stream(stream)))
+        return y
+
+    def launches_per_power_step(self) -> int:
+        return int(lib.yaspmv_launches_per_power_step(self._h))
+
     def spmv_host(self, x: np.ndarray, y: np.ndarray | None = None, stream=None) -> np.ndarray:
         """y := A·x with host arrays (copies in and out inside the call)."""
         x = np.ascontiguousarray(x, dtype=self.dtype)

@@ -41,7 +41,8 @@ def test_remap_is_a_bijection_into_padded_space():
 
 
 class _CpuOps:
-    """Local steps on the CPU for the exchange test (oracle product, fp64 norm)."""
+    """Local steps on the CPU for the exchange test (oracle product, fp64 norm); the
+    unfused protocol (spmv / nrm2sq / scale)."""
 
     def __init__(self, csr):
         self.csr = csr
@@ -57,7 +58,7 @@ class _CpuOps:
         dst.copy_(src / float(np.sqrt(norm2[0].item())))
 
 
-def _worker(rank, world, port, path, n, iters):
+def _worker(rank, world, port, path, n, iters, fused=False):
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -70,11 +71,12 @@ def _worker(rank, world, port, path, n, iters):
     L = D.make_layout(rp, rank, world)
     csr = sm.circuit_like_rows(L.r0, L.r1, **kw)        # only this rank's rows
     csr.col = D.remap_columns(csr.col, L.bounds, L.m_max)
-    pit = D.PowerIteration(L, _CpuOps(csr), torch.float32, torch.device("cpu"))
+    ops = _CpuFusedOps(csr) if fused else _CpuOps(csr)
+    pit = D.PowerIteration(L, ops, torch.float32, torch.device("cpu"))
     for _ in range(iters):
         pit.step()
     if rank == 0:
-        np.save(path, D.unpad(pit.x.numpy(), L.bounds, L.m_max))
+        np.save(path, D.unpad(pit.current_x().numpy(), L.bounds, L.m_max))
     dist.destroy_process_group()
 
 
@@ -86,13 +88,27 @@ def _free_port():
     return p
 
 
-@pytest.mark.parametrize("world", [2])
-def test_power_iteration_world2_matches_single_process(world):
+class _CpuFusedOps:
+    """The fused protocol (power_step: z = (A v)/sqrt(in_norm2), out_norm2 = ||z||^2)."""
+
+    def __init__(self, csr):
+        self.csr = csr
+
+    def power_step(self, v, z, in_norm2, out_norm2):
+        yy, _ = ref.spmv(self.csr.row_ptr, self.csr.col, self.csr.val, v.numpy(), with_bound=False)
+        if in_norm2 is not None:
+            yy = yy / np.sqrt(in_norm2[0].item())
+        z.copy_(torch.from_numpy(yy.astype(np.float32)))
+        out_norm2[0] = float(np.sum(z.numpy().astype(np.float64) ** 2))
+
+
+@pytest.mark.parametrize("world,fused", [(2, False), (2, True), (1, True)])
+def test_power_iteration_world2_matches_single_process(world, fused):
     import torch.multiprocessing as mp
     n, iters = 1 << 13, 4
     with tempfile.TemporaryDirectory() as td:
         path = os.path.join(td, "x.npy")
-        mp.spawn(_worker, args=(world, _free_port(), path, n, iters), nprocs=world, join=True)
+        mp.spawn(_worker, args=(world, _free_port(), path, n, iters, fused), nprocs=world, join=True)
         x_dist = np.load(path)
     # single-process fp64 power iteration on the same matrix
     from synth import matrices as sm

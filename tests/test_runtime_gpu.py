@@ -91,3 +91,51 @@ def test_compute_sanitizer(tool, tmp_path):
     assert "SANITIZE-DONE" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
     assert r.returncode == 0, r.stdout[-3000:]
     assert "ERROR SUMMARY: 0 errors" in r.stdout
+
+
+@pytest.mark.parametrize("S", [1, 3])
+def test_fused_power_step(S):
+    """yaspmv_spmv_power: y = (A x)/sqrt(in), out = sum y^2 (fused epilogue / combine)."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    csr = synth.webbase_like(m=300_000, integer=True)
+    A = Matrix.from_synth(csr, device=0, T=16, C=128, S=S)
+    xn = synth.make_x(csr.n, np.float32, "int2", 1)
+    x = torch.from_numpy(xn).cuda()
+    y = torch.empty(csr.m, dtype=torch.float32, device="cuda")
+    out = torch.zeros(1, dtype=torch.float64, device="cuda")
+    inn = torch.tensor([4.0], dtype=torch.float64, device="cuda")      # scale by 1/2: exact
+    ye, _ = ref.spmv(csr.row_ptr, csr.col, csr.val, xn)
+    A.spmv_power(x, y, None, out)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy().astype(np.float64), ye)
+    assert out.item() == float(np.sum(ye ** 2))                         # integers: exact
+    A.spmv_power(x, y, inn, out)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy().astype(np.float64), ye / 2)
+    assert out.item() == float(np.sum((ye / 2) ** 2))
+    # deterministic run to run
+    vals = set()
+    for _ in range(3):
+        A.spmv_power(x, y, inn, out)
+        torch.cuda.synchronize()
+        vals.add(out.item())
+    assert len(vals) == 1
+    A.free()
+
+
+def test_power_iteration_gpu_matches_fp64():
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix, dist as D
+    from synth import matrices as sm
+    n = 1 << 16
+    a = sm.circuit_like_rows(0, n, n=n, n_net=2, net_log2=(10, 12), band=4096)
+    A = Matrix.from_synth(a, device=0, T=16, C=128)
+    L = D.Layout(0, 1, np.array([0, n], dtype=np.int64), n)
+    pit = D.PowerIteration(L, D.GpuOps(A, n, torch.device("cuda")), torch.float32, torch.device("cuda"))
+    x = np.full(n, 1.0 / np.sqrt(n))
+    for _ in range(6):
+        pit.step()
+        y, _ = ref.spmv(a.row_ptr, a.col, a.val.astype(np.float64), x, with_bound=False)
+        x = y / np.linalg.norm(y)
+    torch.cuda.synchronize()
+    assert np.allclose(pit.current_x().cpu().numpy(), x, rtol=1e-4, atol=1e-7)
+    A.free()

@@ -18,6 +18,7 @@ def main():
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--flush", action="store_true", help="write 2x L2 between launches")
     ap.add_argument("--persist", type=int, default=-1, help="cudaLimitPersistingL2CacheSize in MB (-1: leave)")
+    ap.add_argument("--power", action="store_true", help="time yaspmv_spmv_power (fused epilogue)")
     args = ap.parse_args()
     import torch
 
@@ -52,14 +53,17 @@ def main():
         except Exception as e:
             print(json.dumps({"params": p, "error": str(e)}), flush=True)
             continue
+        n2a = torch.ones(1, dtype=torch.float64, device="cuda")
+        n2b = torch.zeros(1, dtype=torch.float64, device="cuda")
+        call = (lambda: A.spmv_power(x, y, n2a, n2b)) if args.power else (lambda: A.spmv(x, y))
         for _ in range(3):
-            A.spmv(x, y)
+            call()
         ts = []
         for _ in range(args.iters):
             if args.flush:
                 scratch.zero_()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(); A.spmv(x, y); b.record()
+            a.record(); call(); b.record()
             torch.cuda.synchronize()
             ts.append(a.elapsed_time(b))
         info = A.info()
