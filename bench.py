@@ -239,7 +239,8 @@ def main():
     if args.params:
         params.update(json.loads(args.params))
     big = csr.nnz > 50_000_000
-    params.setdefault("flags", 2 if big else 0)  # DROP_CSR for the 1B-nnz matrix
+    # DROP_CSR (no host copy kept) + GPU translation to BCCOO for the 1B-nnz matrix
+    params.setdefault("flags", (2 | 4) if big else 0)
     A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=local_rank, **params)
     info = A.info()
     t_build = time.perf_counter() - t_build0

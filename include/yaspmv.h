@@ -49,7 +49,8 @@ enum { YASPMV_EMPTY_AUTO = 0, YASPMV_EMPTY_FILLER = 1, YASPMV_EMPTY_MAP = 2 };
 /* yaspmv_params.flags */
 enum {
   YASPMV_KEEP_HOST = 1, /* keep the canonical host arrays for yaspmv_export              */
-  YASPMV_DROP_CSR = 2   /* free the normalised host CSR after upload (no tune/reencode)  */
+  YASPMV_DROP_CSR = 2,  /* free the normalised host CSR after upload (no tune/reencode)  */
+  YASPMV_GPU_ENCODE = 4 /* translate to BCCOO/BCCOO+ on the GPU; no host arrays   */
 };
 
 /* Tunable parameters, Table 1.  0 in any field = auto/default. */
@@ -61,7 +62,7 @@ typedef struct {
   int32_t cta_size;    /* C in {64,128,256,512}: threads per workgroup           */
   int32_t col_mode;    /* YASPMV_COL_*; U16 requires ceil(n/w) < 65535           */
   int32_t empty_mode;  /* YASPMV_EMPTY_*                                                  */
-  int32_t flags;       /* YASPMV_KEEP_HOST | YASPMV_DROP_CSR                             */
+  int32_t flags;       /* YASPMV_KEEP_HOST | YASPMV_DROP_CSR | YASPMV_GPU_ENCODE         */
 } yaspmv_params;
 
 typedef struct {

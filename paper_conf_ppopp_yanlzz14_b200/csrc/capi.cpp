@@ -15,6 +15,12 @@
 using namespace yaspmv;
 
 namespace yaspmv {
+void GpuArrays::free_all() {
+  void* ps[] = {val[0], val[1], val[2], val[3], col, col32, flags, cta_seg0, seg_row, zero_rows};
+  for (void* p : ps)
+    if (p) cudaFree(p);
+  *this = GpuArrays();
+}
 static thread_local std::string g_err;
 void set_error(const std::string& msg) { g_err = msg; }
 yaspmv_status fail(yaspmv_status st, const std::string& msg) {
@@ -90,6 +96,19 @@ yaspmv_status upload_permuted(const uint8_t* src, int64_t ntiles, int C, int ptb
   return YASPMV_OK;
 }
 
+// Per-call scratch of an encoding: ticket counter, status words + carries, BCCOO+ buffer.
+yaspmv_status alloc_scratch(const Canonical& c, int vsize, DevArrays& d) {
+  const Params& p = c.p;
+  CUDA_TRY(cudaMalloc((void**)&d.ticket, sizeof(unsigned long long)));
+  CUDA_TRY(cudaMemset(d.ticket, 0, sizeof(unsigned long long)));
+  const int64_t nt = std::max<int64_t>(c.ntiles, 1);
+  CUDA_TRY(cudaMalloc((void**)&d.status, nt * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMemset(d.status, 0, nt * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMalloc((void**)&d.carry, nt * p.h * sizeof(double)));
+  if (p.S > 1) CUDA_TRY(cudaMalloc(&d.tmp, (size_t)p.S * c.MB * p.h * vsize));
+  return YASPMV_OK;
+}
+
 // Encoded host arrays -> a fresh set of device arrays in the device layout.
 yaspmv_status to_device_impl(const Canonical& c, int vsize, DevArrays& d, int64_t& n_escapes) {
   const Params& p = c.p;
@@ -110,13 +129,7 @@ yaspmv_status to_device_impl(const Canonical& c, int vsize, DevArrays& d, int64_
   if ((st = upload(c.cta_seg0.data(), c.cta_seg0.size() * 4, &d.cta_seg0)) != YASPMV_OK) return st;
   if ((st = upload(c.seg_row.data(), c.seg_row.size() * 4, &d.seg_row)) != YASPMV_OK) return st;
   if ((st = upload(c.zero_rows.data(), c.zero_rows.size() * 4, &d.zero_rows)) != YASPMV_OK) return st;
-  CUDA_TRY(cudaMalloc((void**)&d.ticket, sizeof(unsigned long long)));
-  CUDA_TRY(cudaMemset(d.ticket, 0, sizeof(unsigned long long)));
-  const int64_t nt = std::max<int64_t>(c.ntiles, 1);
-  CUDA_TRY(cudaMalloc((void**)&d.status, nt * sizeof(unsigned long long)));
-  CUDA_TRY(cudaMemset(d.status, 0, nt * sizeof(unsigned long long)));
-  CUDA_TRY(cudaMalloc((void**)&d.carry, nt * p.h * sizeof(double)));
-  if (p.S > 1) CUDA_TRY(cudaMalloc(&d.tmp, (size_t)p.S * c.MB * p.h * vsize));
+  if ((st = alloc_scratch(c, vsize, d)) != YASPMV_OK) return st;
   // escapes of the int16 delta column array (only they read col32)
   n_escapes = 0;
   if (p.col_mode == COL_DELTA)
@@ -204,6 +217,44 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
   if (st != YASPMV_OK) return st;
   if (A->device >= 0 && !find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode))
     return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for this (dtype, h, w, T): values per thread > 512 B");
+  if ((p.flags & YASPMV_GPU_ENCODE) && A->device >= 0) {
+    CUDA_TRY(cudaSetDevice(A->device));
+    Canonical meta;
+    GpuArrays g;
+    int64_t esc = 0;
+    if ((st = encode_gpu(A->csr, p, meta, g, esc, nullptr)) != YASPMV_OK) return st;
+    DevArrays nd;
+    for (int r = 0; r < 4; ++r) nd.val[r] = g.val[r];
+    nd.col = g.col;
+    nd.col32 = g.col32;
+    nd.flags = g.flags;
+    nd.cta_seg0 = g.cta_seg0;
+    nd.seg_row = g.seg_row;
+    nd.zero_rows = g.zero_rows;
+    if ((st = alloc_scratch(meta, A->vsize, nd)) != YASPMV_OK) {
+      nd.free_all();
+      return st;
+    }
+    Canonical old;
+    std::swap(old, A->can);
+    A->can = std::move(meta);
+    const KernelEntry* oldk = A->kern;
+    const int64_t oldgrid = A->grid;
+    if ((st = select_kernel(A)) != YASPMV_OK) {
+      nd.free_all();
+      A->can = std::move(old);
+      A->kern = oldk;
+      A->grid = oldgrid;
+      return st;
+    }
+    CUDA_TRY(cudaDeviceSynchronize());
+    A->d.free_all();
+    A->d = nd;
+    A->n_escapes = esc;
+    A->have_host_arrays = false;
+    A->build_s = now_s() - t0;
+    return YASPMV_OK;
+  }
   Canonical c;
   if ((st = encode(A->csr, p, c)) != YASPMV_OK) return st;
   if ((st = install_canonical_impl(A, std::move(c), p.flags)) != YASPMV_OK) return st;

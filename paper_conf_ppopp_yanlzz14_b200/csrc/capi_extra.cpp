@@ -229,23 +229,31 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
     for (int S : Ss) {
       if (S > std::max<int64_t>(NB, 1)) continue;
       for (int cm : cms) {
-        // one encode per (h, w, S, col mode) at the largest tile; (T, C) variants derive
+        // host: one encode per (h, w, S, col mode) at the largest tile, (T, C) variants
+        // derived; GPU translation: a full encode per candidate on the device
+        const bool gpu = (saved.flags & YASPMV_GPU_ENCODE) != 0;
         Params bp0;
         bp0.h = sh.h; bp0.w = sh.w; bp0.S = S; bp0.T = 32; bp0.C = 512; bp0.col_mode = cm;
         bp0.empty_mode = saved.empty_mode;
         Params rp;
         if (resolve_params(bp0, M.m, M.n, rp) != YASPMV_OK) continue;
         Canonical base;
-        if (encode(M, rp, base) != YASPMV_OK) continue;
+        if (!gpu && encode(M, rp, base) != YASPMV_OK) continue;
+        const int64_t nnzb_est = gpu ? count_blocks(M, sh.h, sh.w) : base.nnzb;
         for (int T : {4, 8, 16, 32}) {
           if (!find_kernel(A->dtype, sh.h, sh.w, T, cm)) continue;
           for (int C : {64, 128, 256, 512}) {
             // occupancy bound: at least 2 tiles per SM unless the tile is small
-            const int64_t tiles = (base.nnzb + (int64_t)T * C - 1) / ((int64_t)T * C);
+            const int64_t tiles = (nnzb_est + (int64_t)T * C - 1) / ((int64_t)T * C);
             if (tiles < 2 * sms && (T * C) > 1024) continue;
-            Canonical cand;
-            if (derive_tc(base, T, C, cand) != YASPMV_OK) continue;
-            if (install_canonical(A, std::move(cand), 0) != YASPMV_OK) continue;  // e.g. launch bound
+            if (gpu) {
+              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode, YASPMV_GPU_ENCODE};
+              if (yaspmv_reencode(A, &ap) != YASPMV_OK) continue;
+            } else {
+              Canonical cand;
+              if (derive_tc(base, T, C, cand) != YASPMV_OK) continue;
+              if (install_canonical(A, std::move(cand), 0) != YASPMV_OK) continue;  // e.g. launch bound
+            }
             bool ok = true;
             for (int it = 0; it < 3 && ok; ++it) ok = yaspmv_spmv(A, x, y, stream) == YASPMV_OK;
             if (!ok) continue;

@@ -58,6 +58,18 @@ struct Canonical {
   void release_arrays();
 };
 
+// encoded arrays resident on the device, in the device layout (encode_gpu.cu)
+struct GpuArrays {
+  void* val[4] = {nullptr, nullptr, nullptr, nullptr};
+  void* col = nullptr;
+  int32_t* col32 = nullptr;
+  uint8_t* flags = nullptr;
+  int32_t* cta_seg0 = nullptr;
+  int32_t* seg_row = nullptr;
+  int32_t* zero_rows = nullptr;
+  void free_all();
+};
+
 // status helpers ------------------------------------------------------------------
 void set_error(const std::string& msg);
 yaspmv_status fail(yaspmv_status st, const std::string& msg);
@@ -70,6 +82,9 @@ yaspmv_status normalize_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* ri
 yaspmv_status resolve_params(const Params& in, int64_t m, int64_t n, Params& out);
 yaspmv_status encode(const CSR& A, const Params& p, Canonical& out);
 yaspmv_status derive_tc(const Canonical& base, int T, int C, Canonical& out);
+// GPU translation: A is the normalised host CSR, p resolved (empty_mode may be 0)
+yaspmv_status encode_gpu(const CSR& A, const Params& p, Canonical& meta, GpuArrays& out, int64_t& n_escapes,
+                         void* stream);
 // device layout: per workgroup tile, the per-thread byte runs (ptb bytes each) are
 // transposed into chunks of min(16, ptb) bytes so that chunk j of thread t lives at
 // (tile*C*nch + j*C + t) — the offline transpose of PAPER.md P:269-273.

@@ -267,15 +267,17 @@ def test_spmv_host_and_power_helpers():
     A.free()
 
 
-def test_tune_keeps_results():
+@pytest.mark.parametrize("flags", [0, 4])
+def test_tune_keeps_results(flags):
+    """yaspmv_tune (§4): host encode + derived (T, C) variants, or GPU translation."""
     Matrix = _mat()
     csr = synth.config_matrix("c3-cantilever")
     x = synth.make_x(csr.n, np.float32, "uniform", 8)
     y_ref, bound = ref.spmv(csr.row_ptr, csr.col, csr.val, x)
-    A = Matrix.from_synth(csr, device=0)
+    A = Matrix.from_synth(csr, device=0, flags=flags)
     chosen = A.tune()
     info = A.info()
-    assert info["tune_seconds"] > 0 and chosen["block_h"] in (1, 2, 3, 4)
+    assert info["tune_seconds"] > 0 and chosen["block_h"] in (1, 2, 3, 4) and info["tune_candidates"] > 8
     y = A.spmv(torch.from_numpy(x).cuda()).cpu().numpy()
     assert ref.check_tolerance(y, y_ref, bound, np.float32)[0]
     A.free()
