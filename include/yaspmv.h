@@ -56,7 +56,7 @@ enum {
 /* Tunable parameters, Table 1.  0 in any field = auto/default. */
 typedef struct {
   int32_t block_h;     /* h in {1,2,3,4}     (Table 1 "Block height")            */
-  int32_t block_w;     /* w in {1,2,4}       (Table 1 "Block width")             */
+  int32_t block_w;     /* w in {1,2,4} (Table 1 "Block width"); 8 = extension */
   int32_t slices;      /* S >= 1; 1 = BCCOO, > 1 = BCCOO+ (P:307); S <= ceil(n/w) */
   int32_t thread_tile; /* T in {4,8,16,32}: non-zero blocks per thread       */
   int32_t cta_size;    /* C in {64,128,256,512}: threads per workgroup           */
@@ -162,6 +162,10 @@ yaspmv_status yaspmv_host_sync(yaspmv_matrix A);
  * YASPMV_DROP_CSR (then EINVAL).  On failure A keeps its previous parameters.
  * `chosen` (nullable, host) receives the selected parameters. */
 yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen);
+/* yaspmv_tune_ex: mode 0 = yaspmv_tune (the paper's pruned search); mode 1 = exhaustive
+ * over every compiled block shape (the "exhaustive search" the paper compares its tuner
+ * against). */
+yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode);
 
 /* yaspmv_reencode: re-encode A with new parameters (0 fields = keep current). */
 yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params);

@@ -26,7 +26,7 @@ EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv"
             "yaspmv_tune", "yaspmv_reencode", "yaspmv_get_info", "yaspmv_export", "yaspmv_export_device",
             "yaspmv_nrm2sq", "yaspmv_nrm2sq_scratch_bytes", "yaspmv_scale", "yaspmv_last_error",
             "yaspmv_version", "yaspmv_launches_per_spmv", "yaspmv_spmv_host_async", "yaspmv_host_sync",
-            "yaspmv_spmv_power", "yaspmv_launches_per_power_step"]
+            "yaspmv_spmv_power", "yaspmv_launches_per_power_step", "yaspmv_tune_ex"]
 
 
 class Params(ctypes.Structure):
@@ -79,6 +79,7 @@ def _load():
         "yaspmv_spmv": ([H, vp, vp, vp], ctypes.c_int),
         "yaspmv_spmv_host": ([H, vp, vp, vp], ctypes.c_int),
         "yaspmv_tune": ([H, vp, ctypes.POINTER(Params)], ctypes.c_int),
+        "yaspmv_tune_ex": ([H, vp, ctypes.POINTER(Params), i32], ctypes.c_int),
         "yaspmv_reencode": ([H, ctypes.POINTER(Params)], ctypes.c_int),
         "yaspmv_get_info": ([H, ctypes.POINTER(Info)], ctypes.c_int),
         "yaspmv_export": ([H, i32, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),

@@ -173,7 +173,7 @@ yaspmv_status yaspmv_export_device(yaspmv_matrix A, int32_t which, void* dst, in
 }
 
 // ------------------------------------------------------------------ auto-tuner (§4)
-yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) {
+yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "tuning times the kernels: needs a device handle");
   if (!A->have_csr) return fail(YASPMV_EINVAL, "handle was built with YASPMV_DROP_CSR");
@@ -189,7 +189,7 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
   struct Shape { int64_t fp; int h, w; };
   std::vector<Shape> shapes;
   for (int h = 1; h <= 4; ++h)
-    for (int w : {1, 2, 4}) {
+    for (int w : {1, 2, 4, 8}) {
       bool any = false;
       for (int T : {4, 8, 16, 32}) any |= find_kernel(A->dtype, h, w, T, COL_I32) != nullptr;
       if (!any) continue;
@@ -200,7 +200,7 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
   std::sort(shapes.begin(), shapes.end(), [](const Shape& a, const Shape& b) {
     return std::tie(a.fp, a.h, a.w) < std::tie(b.fp, b.h, b.w);
   });
-  if (shapes.size() > 4) shapes.resize(4);
+  if (mode == 0 && shapes.size() > 4) shapes.resize(4);  // P:321 pruning; mode 1 = exhaustive
 
   // (2) candidates: slices only when x is a large share of L2 (BCCOO+ helps x locality,
   // P:154; its temporary buffer costs traffic)
@@ -306,6 +306,10 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) 
     *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags};
   }
   return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen) {
+  return yaspmv_tune_ex(A, stream, chosen, 0);
 }
 
 // ------------------------------------------------------------------ power iteration

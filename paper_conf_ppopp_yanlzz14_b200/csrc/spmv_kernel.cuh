@@ -128,7 +128,11 @@ __device__ __forceinline__ void gather_x(const VT* x, int64_t cb, int64_t n, uin
     const int64_t i0 = cb * W;
     if (i0 + W <= n) {
       if constexpr (W == 2) ldx2(x + i0, pol, xs);
-      else ldx4(x + i0, pol, xs);
+      else if constexpr (W == 4) ldx4(x + i0, pol, xs);
+      else {
+        ldx4(x + i0, pol, xs);
+        ldx4(x + i0 + 4, pol, xs + 4);
+      }
     } else {  // last block column of a matrix whose width is not a multiple of w (Q4)
 #pragma unroll
       for (int c = 0; c < W; ++c) xs[c] = (i0 + c < n) ? ldx(x + i0 + c, pol) : VT(0);
@@ -520,6 +524,7 @@ void reg_h(std::vector<KernelEntry>& R) {
   reg_w<VT, H, 1>(R);
   reg_w<VT, H, 2>(R);
   reg_w<VT, H, 4>(R);
+  reg_w<VT, H, 8>(R);
 }
 
 }  // namespace yaspmv

@@ -131,9 +131,9 @@ class Matrix:
     def host_sync(self) -> None:
         check(lib.yaspmv_host_sync(self._h))
 
-    def tune(self, stream=None) -> dict:
+    def tune(self, stream=None, exhaustive: bool = False) -> dict:
         p = _lib.Params()
-        check(lib.yaspmv_tune(self._h, _stream(stream), ctypes.byref(p)))
+        check(lib.yaspmv_tune_ex(self._h, _stream(stream), ctypes.byref(p), 1 if exhaustive else 0))
         return p.as_dict()
 
     def reencode(self, **params) -> None:

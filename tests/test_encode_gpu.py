@@ -59,7 +59,7 @@ def test_gpu_encoder_grid(seed):
     dt = np.float32 if seed % 2 == 0 else np.float64
     m, n = int(rng.integers(1, 2500)), int(rng.integers(1, 2500))
     a = synth.random_tiny(seed, m=m, n=n, density=float(rng.uniform(0.001, 0.05)), dtype=dt, integer=True)
-    combos = list(itertools.product([1, 2, 3, 4], [1, 2, 4], [4, 8, 16, 32], [64, 128, 256],
+    combos = list(itertools.product([1, 2, 3, 4], [1, 2, 4, 8], [4, 8, 16, 32], [64, 128, 256],
                                     [0, E.COL_I32, E.COL_DELTA], [E.EMPTY_FILLER, E.EMPTY_MAP]))
     for i in rng.choice(len(combos), size=6, replace=False):
         h, w, T, C, cm, em = combos[i]

@@ -39,7 +39,7 @@ def _compare(csr, h, w, S, T, C, cm, em):
 def test_tiny_random_grid(seed):
     a = synth.random_tiny(seed, dtype=np.float64 if seed % 2 else np.float32, integer=seed % 3 != 0)
     rng = np.random.default_rng(seed)
-    combos = list(itertools.product([1, 2, 3, 4], [1, 2, 4], [4, 8, 16, 32], [64, 128],
+    combos = list(itertools.product([1, 2, 3, 4], [1, 2, 4, 8], [4, 8, 16, 32], [64, 128],
                                     [0, E.COL_I32, E.COL_DELTA], [E.EMPTY_FILLER, E.EMPTY_MAP, 0]))
     for i in rng.choice(len(combos), size=20, replace=False):
         h, w, T, C, cm, em = combos[i]

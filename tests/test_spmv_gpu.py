@@ -70,7 +70,7 @@ def test_launch_bound_is_reported():
 
 
 # ----------------------------------------------------------------------------- brute force grid
-GRID = list(itertools.product([1, 2, 3, 4], [1, 2, 4], [4, 8, 16, 32], [64, 128, 256, 512],
+GRID = list(itertools.product([1, 2, 3, 4], [1, 2, 4, 8], [4, 8, 16, 32], [64, 128, 256, 512],
                               [0, E.COL_I32, E.COL_DELTA], [E.EMPTY_FILLER, E.EMPTY_MAP]))
 
 

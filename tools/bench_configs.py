@@ -38,6 +38,7 @@ def main():
     ap.add_argument("--configs", default=",".join(CONFIGS))
     ap.add_argument("--iters", type=int, default=50)
     ap.add_argument("--md", default=None)
+    ap.add_argument("--exhaustive", action="store_true", help="also run the exhaustive search (P:322)")
     args = ap.parse_args()
     import torch
 
@@ -60,6 +61,13 @@ def main():
         ref.spmv(csr.row_ptr, csr.col, csr.val, x_np, with_bound=False)
         t_cpu = time.perf_counter() - t0
         A = Matrix.from_synth(csr, device=0)
+        ex = None
+        if args.exhaustive:  # the paper's tuned-vs-exhaustive comparison
+            A.tune(exhaustive=True)
+            for _ in range(5):
+                A.spmv(x, y)
+            ex = {"params": A.info()["params"], "ms_warm": timed(lambda: A.spmv(x, y), args.iters),
+                  "tune_s": A.info()["tune_seconds"]}
         chosen = A.tune()
         info = A.info()
         for _ in range(5):
@@ -74,7 +82,7 @@ def main():
              "alg_bytes": info["alg_bytes"], "alg_GBs_cold": info["alg_bytes"] / cold / 1e6,
              "frac_of_measured_hbm_cold": info["alg_bytes"] / cold / 1e6 / peak,
              "footprint_MB": info["footprint_bytes"] / 1e6, "parity_ok": ok, "worst_err_over_tol": worst,
-             "oracle_cpu_ms": t_cpu * 1e3, "oracle_threads": ref.num_threads()}
+             "oracle_cpu_ms": t_cpu * 1e3, "oracle_threads": ref.num_threads(), "exhaustive": ex}
         print(json.dumps(r), flush=True)
         rows.append(r)
         A.free()
@@ -88,6 +96,16 @@ def main():
                         f"C={p['cta_size']}, S={p['slices']}, col={p['col_mode']} | {r['tune_s']:.1f} | {r['ms_warm']:.4f} | "
                         f"{r['ms_cold']:.4f} | {r['gflops_cold']:.1f} | {r['alg_GBs_cold']:.0f} | {r['frac_of_measured_hbm_cold']:.3f} | "
                         f"{'ok' if r['parity_ok'] else 'FAIL'} ({r['worst_err_over_tol']:.2g}) | {r['oracle_cpu_ms']:.2f} |\n")
+            if any(r["exhaustive"] for r in rows):
+                f.write("\n### tuned (4 smallest-footprint shapes, P:321) vs exhaustive over all compiled shapes (P:322)\n\n")
+                f.write("| config | tuned params | tuned warm ms | exhaustive params | exhaustive warm ms | exhaustive tune s | tuned/exhaustive time |\n|---|---|---|---|---|---|---|\n")
+                for r in rows:
+                    e = r["exhaustive"]
+                    if not e:
+                        continue
+                    p, q = r["params"], e["params"]
+                    f.write(f"| {r['config']} | {p['block_h']}x{p['block_w']} T={p['thread_tile']} C={p['cta_size']} | {r['ms_warm']:.4f} | "
+                            f"{q['block_h']}x{q['block_w']} T={q['thread_tile']} C={q['cta_size']} | {e['ms_warm']:.4f} | {e['tune_s']:.1f} | {r['ms_warm'] / e['ms_warm']:.3f} |\n")
 
 
 if __name__ == "__main__":
