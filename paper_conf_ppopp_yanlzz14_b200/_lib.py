@@ -26,7 +26,9 @@ EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv"
             "yaspmv_tune", "yaspmv_reencode", "yaspmv_get_info", "yaspmv_export", "yaspmv_export_device",
             "yaspmv_nrm2sq", "yaspmv_nrm2sq_scratch_bytes", "yaspmv_scale", "yaspmv_last_error",
             "yaspmv_version", "yaspmv_launches_per_spmv", "yaspmv_spmv_host_async", "yaspmv_host_sync",
-            "yaspmv_spmv_power", "yaspmv_launches_per_power_step", "yaspmv_tune_ex"]
+            "yaspmv_spmv_power", "yaspmv_launches_per_power_step", "yaspmv_tune_ex",
+            # include/yaspmv_ablation.h
+            "yaspmv_ablation_spmv", "yaspmv_ablation_tree", "yaspmv_ablation_tree_scratch_bytes"]
 
 
 class Params(ctypes.Structure):
@@ -80,6 +82,9 @@ def _load():
         "yaspmv_spmv_host": ([H, vp, vp, vp], ctypes.c_int),
         "yaspmv_tune": ([H, vp, ctypes.POINTER(Params)], ctypes.c_int),
         "yaspmv_tune_ex": ([H, vp, ctypes.POINTER(Params), i32], ctypes.c_int),
+        "yaspmv_ablation_spmv": ([H, i32, vp, vp, vp], ctypes.c_int),
+        "yaspmv_ablation_tree": ([vp, vp, vp, vp, vp, i64, vp, vp, i64, ctypes.c_int, vp, i64, vp], ctypes.c_int),
+        "yaspmv_ablation_tree_scratch_bytes": ([i64], i64),
         "yaspmv_reencode": ([H, ctypes.POINTER(Params)], ctypes.c_int),
         "yaspmv_get_info": ([H, ctypes.POINTER(Info)], ctypes.c_int),
         "yaspmv_export": ([H, i32, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),

@@ -11,6 +11,7 @@
 #include <cstdlib>
 
 #include "handle.hpp"
+#include "../../include/yaspmv_ablation.h"
 
 using namespace yaspmv;
 
@@ -307,7 +308,7 @@ int64_t alg_bytes(const yaspmv_matrix A) {
 }
 
 yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2 = nullptr,
-                       double* out_norm2 = nullptr) {
+                       double* out_norm2 = nullptr, int ablate = 0) {
   const Canonical& c = A->can;
   const Params& p = c.p;
   cudaStream_t cs = (cudaStream_t)stream;
@@ -353,9 +354,25 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   a.epi = 0;
   a.in_norm2 = in_norm2;
   a.part = A->d_part;
+  a.ablate = ablate;
+  a.dep_row = nullptr;
+  if (ablate & ABL_DEFER_CARRY) {
+    if (p.h != 1 || p.S != 1) return fail(YASPMV_EUNSUPPORTED, "ablation variants need h = 1, S = 1");
+    if (A->abl_ntiles < c.ntiles) {
+      if (A->d_dep_row) cudaFree(A->d_dep_row);
+      A->d_dep_row = nullptr;
+      CUDA_TRY(cudaMalloc((void**)&A->d_dep_row, c.ntiles * sizeof(int64_t)));
+      A->abl_ntiles = c.ntiles;
+    }
+    a.dep_row = A->d_dep_row;
+  }
   if (p.S == 1) a.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
   A->kern->launch(a, p.C, A->grid, stream);
   CUDA_TRY(cudaGetLastError());
+  if (ablate & ABL_DEFER_CARRY) {
+    launch_carry_fixup(A->d.status, A->d.carry, A->d_dep_row, c.ntiles, y, A->dtype, stream);
+    CUDA_TRY(cudaGetLastError());
+  }
   if (p.S > 1) {
     launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream, in_norm2, out_norm2 ? A->d_part : nullptr);
     CUDA_TRY(cudaGetLastError());
@@ -524,6 +541,33 @@ int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
   if (!A || A->can.m == 0) return 0;
   if (A->can.ntiles == 0) return 0;  // memset only
   return A->can.p.S > 1 ? 2 : 1;
+}
+
+yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle");
+  if (variant < 1 || variant > 3) return fail(YASPMV_EINVAL, "ablation variant must be 1, 2 or 3");
+  const int ab = variant == 1 ? ABL_DEFER_CARRY : variant == 2 ? ABL_NO_SKIP : 0;
+  return run_spmv(A, x, y, stream, nullptr, nullptr, ab);
+}
+
+int64_t yaspmv_ablation_tree_scratch_bytes(int64_t n_elem) {
+  const int64_t ntiles = (n_elem + 1023) / 1024;
+  return ntiles * (int64_t)(8 + 8 + 8);
+}
+
+yaspmv_status yaspmv_ablation_tree(const int32_t* rows, const uint8_t* flags, const int32_t* tile_seg0,
+                                   const int32_t* col, const void* val, int64_t n_elem, const void* x, void* y,
+                                   int64_t m, yaspmv_dtype dtype, void* scratch, int64_t scratch_bytes, void* stream) {
+  if (n_elem < 0 || m < 0 || (!rows && (!flags || !tile_seg0))) return fail(YASPMV_EINVAL, "bad tree arguments");
+  if (scratch_bytes < yaspmv_ablation_tree_scratch_bytes(n_elem)) return fail(YASPMV_EINVAL, "scratch too small");
+  const int64_t ntiles = (n_elem + 1023) / 1024;
+  unsigned long long* status = static_cast<unsigned long long*>(scratch);
+  double* carry = reinterpret_cast<double*>(status + ntiles);
+  int64_t* dep = reinterpret_cast<int64_t*>(carry + ntiles);
+  int e = launch_tree_segsum(rows, flags, tile_seg0, col, val, n_elem, x, y, m, dtype, status, carry, dep, stream);
+  if (e) return fail(YASPMV_ECUDA, std::string("tree kernel: ") + cudaGetErrorString((cudaError_t)e));
+  return YASPMV_OK;
 }
 
 int32_t yaspmv_launches_per_power_step(yaspmv_matrix A) {

@@ -12,6 +12,8 @@ namespace yaspmv {
 
 enum ColMode { COL_U16 = 1, COL_I32 = 2, COL_DELTA = 3 };
 enum EmptyMode { EMPTY_FILLER = 1, EMPTY_MAP = 2 };
+// ablation switches (Fig. 14); never set by yaspmv_spmv
+enum Ablate { ABL_DEFER_CARRY = 1, ABL_NO_SKIP = 2 };
 
 struct Params {
   int h = 1, w = 1, S = 1, T = 16, C = 256, col_mode = 0, empty_mode = 0, flags = 0;
@@ -117,6 +119,8 @@ struct KArgs {
   int epi;
   const double* in_norm2;
   double* part;
+  int ablate;              // Ablate bits (0 in production)
+  int64_t* dep_row;        // ABL_DEFER_CARRY: per tile, row of the carried segment or -1
 };
 
 typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
@@ -135,6 +139,11 @@ void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, 
                     const double* in_norm2 = nullptr, double* part = nullptr);
 int64_t combine_blocks(int64_t m);
 void launch_sum_f64(const double* v, int64_t n, double* out, double* partials, void* stream);
+void launch_carry_fixup(const unsigned long long* status, const double* carry, const int64_t* dep_row,
+                        int64_t ntiles, void* y, int dtype, void* stream);
+int launch_tree_segsum(const int32_t* rows, const uint8_t* flags, const int32_t* tile_seg0, const int32_t* col,
+                       const void* val, int64_t n_elem, const void* x, void* y, int64_t m, int dtype,
+                       unsigned long long* status, double* carry, int64_t* dep_row, void* stream);
 void launch_nrm2sq(const void* v, int64_t n, int dtype, double* out, double* partials, void* stream);
 int64_t nrm2sq_blocks(int64_t n);
 void launch_scale(const void* src, void* dst, int64_t n, int dtype, const double* norm2, void* stream);

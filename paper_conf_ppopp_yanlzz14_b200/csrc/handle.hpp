@@ -55,6 +55,8 @@ struct yaspmv_matrix_s {
   double* d_part = nullptr;     // power-iteration epilogue: partials of sum y^2
   double* d_scratch = nullptr;  // two-level reduction scratch
   int64_t npart = 0;
+  int64_t* d_dep_row = nullptr;  // ablation: carried segment row per tile
+  int64_t abl_ntiles = 0;
   int64_t n_escapes = 0;
   double build_s = 0, tune_s = 0;
   int tune_candidates = 0;
@@ -76,6 +78,7 @@ struct yaspmv_matrix_s {
       }
       if (s_in) cudaStreamDestroy(s_in);
       if (d_part) cudaFree(d_part);
+      if (d_dep_row) cudaFree(d_dep_row);
       if (d_scratch) cudaFree(d_scratch);
       if (s_out) cudaStreamDestroy(s_out);
       cudaSetDevice(cur);

@@ -260,7 +260,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
   for (int r = 0; r < H; ++r) v[r] = acc[r];
   const unsigned hs_ballot = __ballot_sync(0xffffffffu, hs);
   // lanes 1..31 all hold a stop: every in-warp segment has size 1 -> skip
-  const bool warp_all_stop = (hs_ballot | 1u) == 0xffffffffu;
+  const bool warp_all_stop = (hs_ballot | 1u) == 0xffffffffu && !(a.ablate & ABL_NO_SKIP);
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
     const int f2 = __shfl_up_sync(0xffffffffu, f, d);
@@ -404,6 +404,16 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
     for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
     if (lane == 0) a.part[tile * (NW + 1) + wid] = ss;
     if (t == 0 && !(Fall && tile > 0)) a.part[tile * (NW + 1) + NW] = 0.0;  // no carried segment
+  }
+  if (a.ablate & ABL_DEFER_CARRY) {  // ablation: carries by a second kernel
+    if (t == 0 && !(Fall && tile > 0)) a.dep_row[tile] = -1;
+    if (dependent) {
+#pragma unroll
+      for (int r = 0; r < H; ++r)
+        if (dep_row * H + r < a.out_limit) out[dep_row * H + r] = dep[r];
+      a.dep_row[tile] = dep_row;
+    }
+    return;
   }
   const unsigned dep_ballot = __ballot_sync(0xffffffffu, dependent);
   if (dep_ballot == 0) return;

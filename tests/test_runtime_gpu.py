@@ -139,3 +139,44 @@ def test_power_iteration_gpu_matches_fp64():
     torch.cuda.synchronize()
     assert np.allclose(pit.current_x().cpu().numpy(), x, rtol=1e-4, atol=1e-7)
     A.free()
+
+
+def test_ablation_variants_match():
+    """The Fig. 14 ablation steps (tools/ablation.py) compute the same y."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix, _lib
+    from paper_conf_ppopp_yanlzz14_b200._lib import check, lib
+    csr = synth.webbase_like(m=200_000, integer=True)
+    xn = synth.make_x(csr.n, np.float32, "int2", 2)
+    ye, _ = ref.spmv(csr.row_ptr, csr.col, csr.val, xn)
+    x = torch.from_numpy(xn).cuda()
+    st = torch.cuda.current_stream().cuda_stream
+    outs = []
+    # COO + tree
+    y = torch.zeros(csr.m, dtype=torch.float32, device="cuda")
+    rows = torch.from_numpy(np.repeat(np.arange(csr.m, dtype=np.int32), np.diff(csr.row_ptr))).cuda()
+    col = torch.from_numpy(csr.col).cuda(); val = torch.from_numpy(csr.val).cuda()
+    sb = int(lib.yaspmv_ablation_tree_scratch_bytes(csr.nnz)); scr = torch.empty(sb, dtype=torch.uint8, device="cuda")
+    check(lib.yaspmv_ablation_tree(rows.data_ptr(), None, None, col.data_ptr(), val.data_ptr(), csr.nnz,
+                                   x.data_ptr(), y.data_ptr(), csr.m, _lib.F32, scr.data_ptr(), sb, st))
+    outs.append(y.cpu().numpy())
+    # BCCOO + tree
+    A = Matrix.from_synth(csr, device=0, T=4, C=256, col_mode=2, flags=1)
+    fl = torch.from_numpy(A.export("flags")).cuda(); cb = torch.from_numpy(A.export("col")).cuda()
+    vb = torch.from_numpy(A.export("val0")).cuda(); cs = torch.from_numpy(A.export("cta_seg0")).cuda()
+    nb = A.info()["nnzb_pad"]
+    sb = int(lib.yaspmv_ablation_tree_scratch_bytes(nb)); scr = torch.empty(sb, dtype=torch.uint8, device="cuda")
+    y = torch.zeros(csr.m, dtype=torch.float32, device="cuda")
+    check(lib.yaspmv_ablation_tree(None, fl.data_ptr(), cs.data_ptr(), cb.data_ptr(), vb.data_ptr(), nb,
+                                   x.data_ptr(), y.data_ptr(), csr.m, _lib.F32, scr.data_ptr(), sb, st))
+    outs.append(y.cpu().numpy())
+    A.free()
+    for T, C in ((16, 128), (4, 64)):
+        A = Matrix.from_synth(csr, device=0, T=T, C=C, col_mode=2)
+        for v in (1, 2, 3):
+            y = torch.zeros(csr.m, dtype=torch.float32, device="cuda")
+            check(lib.yaspmv_ablation_spmv(A._h, v, x.data_ptr(), y.data_ptr(), st))
+            outs.append(y.cpu().numpy())
+        A.free()
+    torch.cuda.synchronize()
+    for o in outs:
+        assert np.array_equal(o.astype(np.float64), ye)
