@@ -111,20 +111,21 @@ def measured_peaks():
     return 6650.0, "fallback"
 
 
-def load_matrix(config: str, rank: int, world: int, dtype):
+def load_matrix(config: str, rank: int, world: int, dtype, rows: int = 0):
     """Returns (local CSR, layout) — the rank's nnz-balanced row block, columns remapped to
     the padded all-gather space when world > 1."""
     import synth
     from synth import matrices as sm
     from paper_conf_ppopp_yanlzz14_b200 import dist as D
     if config == "c5":
+        kw = dict(n=rows) if rows else {}
         if world == 1:
-            csr = sm.circuit_like_rows(0, 50_000_000, dtype=dtype)
+            csr = sm.circuit_like_rows(0, rows or 50_000_000, dtype=dtype, **kw)
             L = D.Layout(0, 1, np.array([0, csr.m], dtype=np.int64), csr.m)
             return csr, L
         # global row lengths (cheap pass) -> partition -> generate only this rank's rows
         import ctypes
-        P = sm.c5_params()
+        P = sm.c5_params(**kw)
         counts = np.empty(P.n, dtype=np.int64)
         sm._lib().c5_count(ctypes.byref(P), ctypes.c_int64(0), ctypes.c_int64(P.n),
                             counts.ctypes.data_as(ctypes.c_void_p))
@@ -132,7 +133,7 @@ def load_matrix(config: str, rank: int, world: int, dtype):
         np.cumsum(counts, out=rp[1:])
         del counts
         L = D.make_layout(rp, rank, world)
-        csr = sm.circuit_like_rows(L.r0, L.r1, dtype=dtype)
+        csr = sm.circuit_like_rows(L.r0, L.r1, dtype=dtype, **kw)
     else:
         full = synth.config_matrix(config)
         if world == 1:
@@ -211,6 +212,9 @@ def main():
     ap.add_argument("--params", default=None, help="JSON dict of build parameters")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=20)
+    ap.add_argument("--backend", default="nccl", help="process-group backend for N > 1 (gloo: exchange-path "
+                    "check with several ranks on one GPU; never a performance number)")
+    ap.add_argument("--rows", type=int, default=0, help="C5 only: use the first ROWS rows/cols (checks)")
     args = ap.parse_args()
 
     world = _env_int("WORLD_SIZE", 1)
@@ -225,15 +229,19 @@ def main():
     from paper_conf_ppopp_yanlzz14_b200 import Matrix
     from paper_conf_ppopp_yanlzz14_b200 import dist as D
 
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
+    ngpu = max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local_rank % ngpu)
+    dev = torch.device("cuda", local_rank % ngpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(args.backend)
     dtype_np = np.float64 if args.config in ("c1", "c2-f64", "c3-ship-f64") else np.float32
     tdt = torch.float64 if dtype_np == np.float64 else torch.float32
 
     t_build0 = time.perf_counter()
-    csr, L = load_matrix(args.config, rank, world, dtype_np)
+    csr, L = load_matrix(args.config, rank, world, dtype_np, args.rows)
     t_gen = time.perf_counter() - t_build0
     params = dict(DEFAULT_PARAMS.get(args.config, {}))
     if args.params:
@@ -241,7 +249,7 @@ def main():
     big = csr.nnz > 50_000_000
     # DROP_CSR (no host copy kept) + GPU translation to BCCOO for the 1B-nnz matrix
     params.setdefault("flags", (2 | 4) if big else 0)
-    A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=local_rank, **params)
+    A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=local_rank % ngpu, **params)
     info = A.info()
     t_build = time.perf_counter() - t_build0
 
@@ -258,7 +266,7 @@ def main():
         dist.barrier()
 
     # ---- timed region: K steps, CUDA events on the launching stream ----------------
-    sampler = ClockSampler(local_rank)
+    sampler = ClockSampler(local_rank % ngpu)
     sampler.start()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
