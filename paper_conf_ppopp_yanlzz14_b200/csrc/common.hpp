@@ -120,6 +120,7 @@ struct KArgs {
   const double* in_norm2;
   double* part;
   int ablate;              // Ablate bits (0 in production)
+  int block_ids;           // 1: tile = blockIdx (in-order dispatch), ticket only for the epoch
   int64_t* dep_row;        // ABL_DEFER_CARRY: per tile, row of the carried segment or -1
 };
 

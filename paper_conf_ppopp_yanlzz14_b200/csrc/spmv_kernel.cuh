@@ -173,7 +173,7 @@ struct ScanShared {
 // The work of one workgroup-level tile (T*C consecutive blocks): steps 1-3
 // of P:226 plus the cross-tile carry.
 template <typename VT, int H, int W, int T, int CM, bool EPI>
-__device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, const unsigned long long epoch,
+__device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, const unsigned long long tk,
                                           ScanShared<VT, H>& sh) {
   using TR = KTraits<VT, H, W, T, CM>;
   constexpr int VB = TR::VB, CB = TR::CB;
@@ -291,7 +291,11 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
 #pragma unroll
     for (int r = 0; r < H; ++r) vx[r] = VT(0);
   }
+  // block-id mode (in-order dispatch): the ticket only yields the launch epoch,
+  // needed from here on, so its atomic latency hides behind the tile's loads
+  if (a.block_ids && t == 0) sh.epoch = tk / (unsigned long long)a.period + 1ull;
   __syncthreads();
+  const unsigned long long epoch = sh.epoch;
   int Fw = 0, Nw = 0, Fall = 0;
   VT Vw[H];
 #pragma unroll
@@ -464,7 +468,16 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
 template <typename VT, int H, int W, int T, int CM, bool EPI>
 __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) spmv_bccoo_kernel(const KArgs a) {
   __shared__ ScanShared<VT, H> sh;
-  if (threadIdx.x == 0) {
+  if (a.block_ids) {  // tile = workgroup id: workgroups dispatch in order — the default
+    unsigned long long tk = 0;
+    if (threadIdx.x == 0) {
+      tk = atomicAdd(a.ticket, 1ull);  // consumed only at the scan barrier (epoch)
+      if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
+    }
+    tile_body<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, tk, sh);
+    return;
+  }
+  if (threadIdx.x == 0) {  // logical workgroup id from an atomic ticket
     const unsigned long long tk = atomicAdd(a.ticket, 1ull);
     const unsigned long long q = tk / (unsigned long long)a.period;
     sh.tile = (long long)(tk - q * (unsigned long long)a.period);
@@ -472,7 +485,7 @@ __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) s
     if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   }
   __syncthreads();
-  tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, sh.epoch, sh);
+  tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, 0ull, sh);
 }
 
 template <typename VT, int H, int W, int T, int CM>

@@ -96,7 +96,8 @@ def test_integer_exact_random_grid(seed):
             assert np.array_equal(y.astype(np.float64), y_exact), (h, w, T, C, S, cm, em, info)
 
 
-def test_long_row_spanning_many_ctas():
+@pytest.mark.parametrize("flags", [0, 8])
+def test_long_row_spanning_many_ctas(flags):
     """One row of 600k entries crosses hundreds of workgroup tiles: carries travel through
     the look-back chain (adjacent synchronization)."""
     n = 700_000
@@ -110,7 +111,7 @@ def test_long_row_spanning_many_ctas():
     x = synth.make_x(n, np.float32, "int2", 1)
     ref_y = _dense_exact_rows(csr, x)
     for T, C in ((4, 64), (16, 256), (32, 512)):
-        y, info = _run(csr, x, T=T, C=C, col_mode=E.COL_I32)
+        y, info = _run(csr, x, T=T, C=C, col_mode=E.COL_I32, flags=flags)
         assert info["ntiles"] > 30
         assert np.array_equal(y.astype(np.float64), ref_y)
 
@@ -135,12 +136,22 @@ CONFIG_PARAMS = {
 
 @pytest.mark.parametrize("name", list(CONFIG_PARAMS))
 def test_configs_tolerance(name):
+    _configs_tolerance(name, 0)
+
+
+@pytest.mark.parametrize("name", ["c1", "c3-ship", "c4"])
+def test_configs_tolerance_ticket_ids(name):
+    """YASPMV_TICKET_IDS: logical tile ids from the atomic ticket."""
+    _configs_tolerance(name, 8)
+
+
+def _configs_tolerance(name, flags):
     csr = synth.config_matrix(name)
     dt = csr.val.dtype
     x = synth.make_x(csr.n, dt, "unit" if name == "c4" else "uniform", 3)
     y_ref, bound = ref.spmv(csr.row_ptr, csr.col, csr.val, x)
     for p in CONFIG_PARAMS[name]:
-        y, info = _run(csr, x, **p)
+        y, info = _run(csr, x, flags=flags, **p)
         ok, worst = ref.check_tolerance(y, y_ref, bound, dt)
         assert ok, (name, p, worst)
 

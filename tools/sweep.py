@@ -19,6 +19,7 @@ def main():
     ap.add_argument("--flush", action="store_true", help="write 2x L2 between launches")
     ap.add_argument("--persist", type=int, default=-1, help="cudaLimitPersistingL2CacheSize in MB (-1: leave)")
     ap.add_argument("--power", action="store_true", help="time yaspmv_spmv_power (fused epilogue)")
+    ap.add_argument("--l2fetch", type=int, default=0, help="cudaLimitMaxL2FetchGranularity (32/64/128), 0 = leave")
     args = ap.parse_args()
     import torch
 
@@ -37,6 +38,17 @@ def main():
         got = ctypes.c_size_t()
         rt.cudaDeviceGetLimit(ctypes.byref(got), 0x06)
         print(f"# persisting L2: max {mx.value >> 20} MB, set {want >> 20} MB rc={rc} now {got.value >> 20} MB", flush=True)
+    if args.l2fetch:
+        import ctypes
+        torch.zeros(1, device="cuda")
+        rt = ctypes.CDLL(os.path.join(os.path.dirname(torch.__file__), "..", "nvidia", "cuda_runtime", "lib",
+                                      "libcudart.so.12"))
+        cur = ctypes.c_size_t()
+        rt.cudaDeviceGetLimit(ctypes.byref(cur), 0x05)
+        rc = rt.cudaDeviceSetLimit(0x05, ctypes.c_size_t(args.l2fetch))
+        now = ctypes.c_size_t()
+        rt.cudaDeviceGetLimit(ctypes.byref(now), 0x05)
+        print(f"# L2 fetch granularity: was {cur.value}, set {args.l2fetch} rc={rc}, now {now.value}", flush=True)
     t0 = time.time()
     csr = sm.circuit_like_rows(0, 50_000_000) if args.config == "c5" else synth.config_matrix(args.config)
     print(f"# generated {args.config} nnz={csr.nnz} in {time.time()-t0:.1f}s", flush=True)
