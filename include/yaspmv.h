@@ -51,11 +51,14 @@ enum {
   YASPMV_KEEP_HOST = 1, /* keep the canonical host arrays for yaspmv_export              */
   YASPMV_DROP_CSR = 2,  /* free the normalised host CSR after upload (no tune/reencode)  */
   YASPMV_GPU_ENCODE = 4, /* translate to BCCOO/BCCOO+ on the GPU; no host arrays  */
-  YASPMV_TICKET_IDS = 8  /* take logical tile ids from an atomic ticket (for GPUs
+  YASPMV_TICKET_IDS = 8, /* take logical tile ids from an atomic ticket (for GPUs
                             that dispatch workgroups out of order).  Default: tile =
                             workgroup id, relying on in-order dispatch as the paper does
                             ("Current GPUs dispatch workgroups in-order"); the
                             ticket then only yields the launch epoch                       */
+  YASPMV_NO_PDL = 16     /* launch without programmatic dependent launch (by default each
+                            SpMV may start streaming its matrix tiles while the previous
+                            kernel on the stream drains; x, y and carries wait for it)     */
 };
 
 /* Tunable parameters, Table 1.  0 in any field = auto/default. */

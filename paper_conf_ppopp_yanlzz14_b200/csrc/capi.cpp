@@ -356,6 +356,7 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   a.part = A->d_part;
   a.ablate = ablate;
   a.block_ids = (p.flags & YASPMV_TICKET_IDS) ? 0 : 1;
+  a.pdl = (p.flags & YASPMV_NO_PDL) ? 0 : 1;
   a.dep_row = nullptr;
   if (ablate & ABL_DEFER_CARRY) {
     if (p.h != 1 || p.S != 1) return fail(YASPMV_EUNSUPPORTED, "ablation variants need h = 1, S = 1");

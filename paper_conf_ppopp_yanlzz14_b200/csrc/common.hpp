@@ -121,6 +121,7 @@ struct KArgs {
   double* part;
   int ablate;              // Ablate bits (0 in production)
   int block_ids;           // 1: tile = blockIdx (in-order dispatch), ticket only for the epoch
+  int pdl;                 // launched with programmatic dependent launch
   int64_t* dep_row;        // ABL_DEFER_CARRY: per tile, row of the carried segment or -1
 };
 

@@ -17,6 +17,7 @@ __device__ __forceinline__ double block_sum256(double v);
 template <typename VT>
 __global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, int64_t m, int64_t stride, int S,
                                const double* __restrict__ in_norm2, double* __restrict__ part) {
+  cudaTriggerProgrammaticLaunchCompletion();
   const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
   const double inv = in_norm2 ? 1.0 / sqrt(in_norm2[0]) : 1.0;
   double ss = 0.0;
@@ -101,6 +102,7 @@ __global__ void nrm2sq_partial(const VT* __restrict__ v, int64_t n, double* __re
 __device__ __forceinline__ double block_sum256(double v) { return block_sum(v); }
 
 __global__ void sum_f64_partial(const double* __restrict__ v, int64_t n, double* __restrict__ partials) {
+  cudaTriggerProgrammaticLaunchCompletion();
   double s = 0.0;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) s += v[i];
@@ -109,6 +111,7 @@ __global__ void sum_f64_partial(const double* __restrict__ v, int64_t n, double*
 }
 
 __global__ void nrm2sq_final(const double* __restrict__ partials, int nb, double* __restrict__ out) {
+  cudaTriggerProgrammaticLaunchCompletion();
   double s = 0.0;
   for (int i = threadIdx.x; i < nb; i += blockDim.x) s += partials[i];
   s = block_sum(s);

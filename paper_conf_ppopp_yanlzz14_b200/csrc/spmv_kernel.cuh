@@ -192,8 +192,7 @@ struct ScanShared {
 // The work of one workgroup-level tile (T*C consecutive blocks): steps 1-3
 // of P:226 plus the cross-tile carry.
 template <typename VT, int H, int W, int T, int CM, bool EPI>
-__device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, const unsigned long long tk,
-                                          ScanShared<VT, H>& sh) {
+__device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, ScanShared<VT, H>& sh) {
   using TR = KTraits<VT, H, W, T, CM>;
   constexpr int VB = TR::VB, CB = TR::CB;
   constexpr uint32_t TMASK = (T == 32) ? 0xffffffffu : ((1u << T) - 1u);
@@ -214,6 +213,17 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
   for (int r = 0; r < H; ++r) dev::load_run<VB>(a.val[r], tile, C, t, pol_s, vw[r]);
 
   VT* out = static_cast<VT*>(a.out);
+  // Programmatic dependent launch: everything above reads only the encoded matrix (never
+  // written by other kernels) and overlaps the previous kernel's tail; x, y, the status
+  // words and the ticket may depend on earlier kernels in the stream.
+  unsigned long long tk = 0;
+  if (a.block_ids) {
+    if (a.pdl) cudaGridDependencySynchronize();
+    if (t == 0) {
+      tk = atomicAdd(a.ticket, 1ull);  // consumed only at the scan barrier (epoch)
+      if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
+    }
+  }
   // zero-fill of stacked rows that hold no block (empty_mode MAP, Q1)
   if (a.n_zero > 0) {
     const int64_t per = (a.n_zero + a.ntiles - 1) / a.ntiles;
@@ -487,15 +497,12 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, co
 template <typename VT, int H, int W, int T, int CM, bool EPI>
 __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) spmv_bccoo_kernel(const KArgs a) {
   __shared__ ScanShared<VT, H> sh;
+  if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();  // the next SpMV may start its loads
   if (a.block_ids) {  // tile = workgroup id: workgroups dispatch in order — the default
-    unsigned long long tk = 0;
-    if (threadIdx.x == 0) {
-      tk = atomicAdd(a.ticket, 1ull);  // consumed only at the scan barrier (epoch)
-      if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
-    }
-    tile_body<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, tk, sh);
+    tile_body<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, sh);
     return;
   }
+  if (a.pdl) cudaGridDependencySynchronize();
   if (threadIdx.x == 0) {  // logical workgroup id from an atomic ticket
     const unsigned long long tk = atomicAdd(a.ticket, 1ull);
     const unsigned long long q = tk / (unsigned long long)a.period;
@@ -504,14 +511,24 @@ __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) s
     if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   }
   __syncthreads();
-  tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, 0ull, sh);
+  tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, sh);
 }
 
 template <typename VT, int H, int W, int T, int CM>
 void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
   using TR = KTraits<VT, H, W, T, CM>;
-  if (a.epi) spmv_bccoo_kernel<VT, H, W, T, CM, true><<<(unsigned)grid, C, TR::smem_bytes(C), (cudaStream_t)stream>>>(a);
-  else spmv_bccoo_kernel<VT, H, W, T, CM, false><<<(unsigned)grid, C, TR::smem_bytes(C), (cudaStream_t)stream>>>(a);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(C);
+  cfg.dynamicSmemBytes = TR::smem_bytes(C);
+  cfg.stream = (cudaStream_t)stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (a.epi) cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, true>, a);
+  else cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, false>, a);
 }
 
 template <typename VT, int H, int W, int T, int CM>

@@ -47,6 +47,28 @@ def test_cuda_graph_replay():
     A.free()
 
 
+@pytest.mark.parametrize("flags", [0, 16, 8, 8 | 16])
+@pytest.mark.parametrize("S,empty", [(1, 2), (2, 1)])
+def test_back_to_back_chain(flags, S, empty):
+    """Dependent SpMVs queued without a host sync (x_{k+1} = A x_k, ping-pong buffers):
+    with programmatic dependent launch (default) the next launch streams its matrix tiles
+    while the previous drains, but x, y, the zero-fill and the carries wait for it.
+    Exact on an integer f64 matrix (|A x| stays far below 2^53)."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    csr = synth.webbase_like(m=300_000, dtype=np.float64, integer=True)
+    A = Matrix.from_synth(csr, device=0, T=8, C=128, S=S, empty_mode=empty, flags=flags)
+    x0 = synth.make_x(csr.n, np.float64, "int2", 5)
+    buf = [torch.from_numpy(x0).cuda(), torch.empty(csr.m, dtype=torch.float64, device="cuda")]
+    for k in range(4):
+        A.spmv(buf[k % 2], buf[(k + 1) % 2])
+    torch.cuda.synchronize()
+    ye = x0
+    for k in range(4):
+        ye, _ = ref.spmv(csr.row_ptr, csr.col, csr.val, ye)
+    assert np.array_equal(buf[0].cpu().numpy(), ye)
+    A.free()
+
+
 def test_host_async_pipeline():
     from paper_conf_ppopp_yanlzz14_b200 import Matrix
     csr = synth.fem_like("cantilever", integer=True)

@@ -33,6 +33,20 @@ def timed(fn, iters, flush=None):
     return float(np.median(ts))
 
 
+def timed_b2b(fn, n=100):
+    """Steady-state time per launch of n back-to-back launches (one event pair)."""
+    import torch
+    for _ in range(5):
+        fn()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(n):
+        fn()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / n
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", default=",".join(CONFIGS))
@@ -74,10 +88,17 @@ def main():
             A.spmv(x, y)
         warm = timed(lambda: A.spmv(x, y), args.iters)
         cold = timed(lambda: A.spmv(x, y), max(10, args.iters // 5), flush)
+        b2b = timed_b2b(lambda: A.spmv(x, y))
         ok, worst = ref.check_tolerance(y.cpu().numpy(), y_ref, bound, dt)
+        # the same tuned parameters launched without programmatic dependent launch
+        q = {k: v for k, v in chosen.items()}
+        B = Matrix.from_synth(csr, device=0, h=q["block_h"], w=q["block_w"], S=q["slices"], T=q["thread_tile"],
+                              C=q["cta_size"], col_mode=q["col_mode"], empty_mode=q["empty_mode"], flags=16)
+        b2b_nopdl = timed_b2b(lambda: B.spmv(x, y))
+        B.free()
         r = {"config": name, "m": csr.m, "nnz": csr.nnz, "dtype": str(dt), "params": chosen,
              "tune_s": info["tune_seconds"], "tune_candidates": info["tune_candidates"],
-             "ms_warm": warm, "ms_cold": cold,
+             "ms_warm": warm, "ms_cold": cold, "ms_b2b": b2b, "ms_b2b_no_pdl": b2b_nopdl,
              "gflops_warm": 2 * csr.nnz / warm / 1e6, "gflops_cold": 2 * csr.nnz / cold / 1e6,
              "alg_bytes": info["alg_bytes"], "alg_GBs_cold": info["alg_bytes"] / cold / 1e6,
              "frac_of_measured_hbm_cold": info["alg_bytes"] / cold / 1e6 / peak,
@@ -88,13 +109,13 @@ def main():
         A.free()
     if args.md:
         with open(args.md, "w") as f:
-            f.write("| config | nnz | dtype | tuned (h,w,T,C,S,col) | tune s | warm ms | cold ms | GFLOPS (cold) | alg GB/s (cold) | frac of measured HBM | parity (worst err/tol) | oracle CPU ms |\n")
-            f.write("|---|---|---|---|---|---|---|---|---|---|---|---|\n")
+            f.write("| config | nnz | dtype | tuned (h,w,T,C,S,col) | tune s | warm ms | cold ms | back-to-back ms (no PDL) | GFLOPS (cold) | alg GB/s (cold) | frac of measured HBM | parity (worst err/tol) | oracle CPU ms |\n")
+            f.write("|---|---|---|---|---|---|---|---|---|---|---|---|---|\n")
             for r in rows:
                 p = r["params"]
                 f.write(f"| {r['config']} | {r['nnz']:,} | {r['dtype']} | {p['block_h']}x{p['block_w']}, T={p['thread_tile']}, "
                         f"C={p['cta_size']}, S={p['slices']}, col={p['col_mode']} | {r['tune_s']:.1f} | {r['ms_warm']:.4f} | "
-                        f"{r['ms_cold']:.4f} | {r['gflops_cold']:.1f} | {r['alg_GBs_cold']:.0f} | {r['frac_of_measured_hbm_cold']:.3f} | "
+                        f"{r['ms_cold']:.4f} | {r['ms_b2b']:.4f} ({r['ms_b2b_no_pdl']:.4f}) | {r['gflops_cold']:.1f} | {r['alg_GBs_cold']:.0f} | {r['frac_of_measured_hbm_cold']:.3f} | "
                         f"{'ok' if r['parity_ok'] else 'FAIL'} ({r['worst_err_over_tol']:.2g}) | {r['oracle_cpu_ms']:.2f} |\n")
             if any(r["exhaustive"] for r in rows):
                 f.write("\n### tuned (4 smallest-footprint shapes, P:321) vs exhaustive over all compiled shapes (P:322)\n\n")
