@@ -215,6 +215,10 @@ def main():
     ap.add_argument("--backend", default="nccl", help="process-group backend for N > 1 (gloo: exchange-path "
                     "check with several ranks on one GPU; never a performance number)")
     ap.add_argument("--rows", type=int, default=0, help="C5 only: use the first ROWS rows/cols (checks)")
+    ap.add_argument("--exchange", default="auto", choices=["auto", "fused", "nccl"],
+                    help="x replication for N > 1: fused = SpMV write-back into every rank's x over peer "
+                         "memory (yaspmv_power_step_fused, CUDA IPC); nccl = all_reduce + all_gather_into_tensor. "
+                         "auto: fused for N > 1 (nccl if IPC mapping fails), none for N = 1")
     args = ap.parse_args()
 
     world = _env_int("WORLD_SIZE", 1)
@@ -256,11 +260,31 @@ def main():
     ops = D.GpuOps(A, L.m_local, dev)
     if args.config != "c5" and csr.m != csr.n and world == 1:
         raise SystemExit("power iteration needs a square matrix")
-    pit = D.PowerIteration(L, ops, tdt, dev)
     stream = torch.cuda.current_stream()
+    exchange = args.exchange
+    if exchange == "auto":
+        exchange = "fused" if world > 1 else "none"
+    fpit = None
+    if exchange == "fused":
+        try:
+            fpit = D.FusedPowerIteration(L, A, tdt, dev, timeout_ms=120000)
+        except Exception as e:  # e.g. no P2P/IPC between the GPUs: the NCCL protocol instead
+            if args.exchange == "fused":
+                raise
+            print(f"[bench] fused exchange unavailable ({e}); using NCCL", file=sys.stderr)
+            exchange = "nccl"
+    if exchange == "none" and world > 1:
+        exchange = "nccl"
+    pit = D.PowerIteration(L, ops, tdt, dev) if fpit is None else None
+
+    def one_step():
+        if fpit is not None:
+            fpit.step(stream)
+        else:
+            pit.step()
 
     for _ in range(max(args.warmup, 3)):
-        pit.step()
+        one_step()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -276,6 +300,13 @@ def main():
     e0.record(stream)
     L_ = L
     for k in range(args.steps):
+        if fpit is not None:
+            # fused exchange: wait for the peers' previous step + SpMV storing z_k into every
+            # rank's x + ||z_k||^2 + publish; the events bracket the whole step
+            ev[k][0].record(stream)
+            fpit.step(stream)
+            ev[k][1].record(stream)
+            continue
         # the fused step: SpMV kernel with the 1/||z_{k-1}|| scaling and ||z_k||^2 partials in
         # its epilogue (+ 2 tiny reduction kernels); events bracket it on the launching stream
         ev[k][0].record(stream)
@@ -288,8 +319,12 @@ def main():
         else:
             pit.x, pit.y = pit.y, pit.x
         pit.norm_prev, pit.norm2 = pit.norm2, pit.norm_prev
+    if fpit is not None:
+        fpit.comm.wait(stream)  # every peer's last step is complete
     e1.record(stream)
     torch.cuda.synchronize()
+    if fpit is not None:
+        fpit.comm.check()
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
@@ -313,7 +348,8 @@ def main():
     # every step copies x host->device and y device->host; yaspmv_spmv_host_async overlaps
     # the copies of consecutive steps with the SpMV (two buffer slots, two copy streams)
     xh = torch.empty(L.n_padded, dtype=tdt).pin_memory()
-    xh.copy_(pit.current_x().cpu())
+    x_cur = fpit.current_x(stream) if fpit is not None else pit.current_x()
+    xh.copy_(x_cur.cpu())
     yh = torch.empty(L.m_local, dtype=tdt).pin_memory()
     A.spmv_host_async(xh.numpy(), yh.numpy(), stream=stream.cuda_stream)
     A.host_sync()
@@ -350,11 +386,16 @@ def main():
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f32" if dtype_np == np.float32 else "f64", "data": "synthetic",
             "config": {"workload": args.config, "m": int(L.bounds[-1]), "nnz": int(nnz_total),
-                       "params": info["params"], "parallelism": f"row-partition x{world}, NCCL all-gather of x",
+                       "params": info["params"],
+                       "parallelism": f"row-partition x{world}" + (
+                           ", x replicated by peer stores from the SpMV epilogue (CUDA IPC over NVLink)"
+                           if fpit is not None else ", NCCL all-gather of x" if world > 1 else ""),
                        "l2": "inputs larger than L2 (matrix 8.5 GB vs 126 MB L2), no flush" if args.config == "c5"
                        else "L2-resident workload; back-to-back steps (warm L2)",
                        "step": "z_k = A z_{k-1}/||z_{k-1}|| and ||z_k||^2 in one fused BCCOO SpMV launch (+2 tiny sums)"
-                               + (" + NCCL allreduce(1 fp64) + allgather(z)" if world > 1 else "")},
+                               + (" + NCCL allreduce(1 fp64) + allgather(z)" if world > 1 and fpit is None else "")
+                               + (" storing z_k into every rank's x (peer memory) + publish/wait kernels"
+                                  if fpit is not None else "")},
             "spmv_ms": spmv_ms, "spmv_ms_max_over_ranks": spmv_ms_max,
             "spmv_gflops": 2.0 * info["nnz"] / (spmv_ms * 1e-3) / 1e9,
             "hbm_gbs_alg": achieved, "pct_of_8TBs": achieved / 8000.0 * 100.0,
@@ -363,17 +404,22 @@ def main():
                          "kernel": "spmv_bccoo_kernel" + (" + combine" if info["params"]["slices"] > 1 else "")
                                    + " (+ 2 tiny y^2-partial reductions of the fused step)",
                          "alg_bytes_per_launch": info["alg_bytes"]},
-            "gpu_launches": A.launches_per_power_step() * args.steps,
+            "gpu_launches": (fpit.launches_per_step() if fpit is not None else A.launches_per_power_step())
+                            * args.steps,
             "clocks": clocks, "e2e": e2e,
             "build": {"generate_s": t_gen, "build_s": t_build, "encode_upload_s": info["build_seconds"]},
         }
         if world == 1 and not args.no_cpu_baseline:
-            x_np = pit.current_x()[: L.m_local].cpu().numpy().astype(dtype_np)
+            x_np = x_cur[: L.m_local].cpu().numpy().astype(dtype_np)
             if args.config == "c5":
                 line["cpu_baseline"] = cpu_baseline(csr, x_np)
             else:
                 line["cpu_baseline"] = cpu_baseline(csr, x_np)
         print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()  # no rank frees its comm while a peer may still map it
+    if fpit is not None:
+        fpit.comm.free()
     A.free()
     if world > 1:
         dist.destroy_process_group()

@@ -217,6 +217,69 @@ int64_t yaspmv_nrm2sq_scratch_bytes(int64_t n);
 yaspmv_status yaspmv_scale(const void* src, void* dst, int64_t n, yaspmv_dtype dtype, const double* norm2_dev,
                            void* stream);
 
+/* ---------------------------------------------------------------- fused multi-GPU power step
+ * Iterated SpMV with A row-partitioned over P ranks (one process or one handle per GPU)
+ * and x replicated (BASELINE.json north_star; not in the
+ * paper, whose method is single-GPU).  Instead of "SpMV, then an all-gather of y"
+ * the SpMV's write-back stores every finished row of z_k straight into ALL ranks' copies of
+ * the next x over peer memory (NVLink P2P stores through CUDA IPC mappings), tile by tile,
+ * so the exchange overlaps the SpMV; a one-warp publish kernel then posts the rank's
+ * ||z_k||^2 partial and an epoch flag into every peer's signal pad (system-scope release),
+ * and the next step's one-warp wait kernel acquires all P flags before x is read.
+ *
+ * A yaspmv_comm owns ONE device allocation on its rank's device (so one IPC handle maps it):
+ *   xbuf[2][n_padded] of dtype   the replicated x, double-buffered by step parity
+ *   signal pad                    per source rank: epoch flag (u64), ||z||^2 partials (f64)[2]
+ * Rank r's rows are the padded chunk [r*chunk, r*chunk + m_r) of x (dist.remap_columns
+ * maps the matrix columns into that padded space; pad entries are zero and never read).
+ *
+ * Protocol (all ranks call the same sequence; seq = steps issued on this comm so far):
+ *   yaspmv_comm_create          on every rank;
+ *   yaspmv_comm_ipc_handle      -> exchange the 64-byte handles (e.g. torch all_gather_object)
+ *   yaspmv_comm_open_ipc        maps every peer (cudaIpcMemLazyEnablePeerAccess), or
+ *   yaspmv_comm_connect_local   same-process peers (tests: P ranks as P handles on 1 GPU);
+ *   write x_0 (replicated) into yaspmv_comm_x(c, 0) on every rank, yaspmv_comm_begin(c),
+ *   then a host barrier across ranks (every rank's x_0 and peers' buffers ready);
+ *   yaspmv_power_step_fused     repeatedly: step k reads xbuf[k%2] (z_{k-1}, or x_0 right
+ *                               after begin) and computes z_k = A_r x / ||z_{k-1}|| (no
+ *                               scaling right after begin) into every rank's xbuf[(k+1)%2];
+ *                               for k after begin it first waits (on the device) for every
+ *                               peer's step k-1;
+ *   yaspmv_comm_wait            waits for every peer's latest step and writes the total
+ *                               ||z||^2 (fp64, summed in rank order: identical on all ranks)
+ *                               into the device double yaspmv_comm_norm2_device(c).
+ * Deterministic: bitwise identical to running yaspmv_spmv_power per rank on the gathered x
+ * with the norms summed in rank order.  The device waits time out after `timeout_ms`
+ * (yaspmv_comm_create; 0 = 60 s): the wait kernel then gives up, and the next
+ * yaspmv_comm_check reports YASPMV_ECUDA instead of hanging the GPU.
+ * A comm and the matrices stepped with it must live on the same device; A's column count
+ * must equal n_padded, A's row count must be <= chunk.  world <= YASPMV_MAX_RANKS. */
+#define YASPMV_MAX_RANKS 8
+typedef struct yaspmv_comm_s* yaspmv_comm;
+yaspmv_status yaspmv_comm_create(int32_t device, int32_t rank, int32_t world, int64_t chunk, yaspmv_dtype dtype,
+                                 int32_t timeout_ms, yaspmv_comm* out);
+/* out: host buffer of >= 64 bytes (a cudaIpcMemHandle_t of the comm's allocation). */
+yaspmv_status yaspmv_comm_ipc_handle(yaspmv_comm c, void* out, int64_t bytes);
+/* handles: host, world * 64 bytes, rank order (this rank's own entry is ignored). */
+yaspmv_status yaspmv_comm_open_ipc(yaspmv_comm c, const void* handles, int64_t bytes);
+/* peers: host array of `world` comms of this process on the same device, rank order. */
+yaspmv_status yaspmv_comm_connect_local(yaspmv_comm c, const yaspmv_comm* peers, int32_t world);
+/* device pointer of x buffer (seq + which) % 2: which = 0 is the next step's input (after a
+ * completed step: the latest z), 1 the buffer the next step writes. */
+void* yaspmv_comm_x(yaspmv_comm c, int32_t which);
+/* the next step reads x_0 unscaled and does not wait for peers (see the protocol). */
+yaspmv_status yaspmv_comm_begin(yaspmv_comm c);
+yaspmv_status yaspmv_power_step_fused(yaspmv_matrix A, yaspmv_comm c, void* stream);
+yaspmv_status yaspmv_comm_wait(yaspmv_comm c, void* stream);
+double* yaspmv_comm_norm2_device(yaspmv_comm c);
+int64_t yaspmv_comm_seq(yaspmv_comm c);
+/* reports (and clears) a device-side wait timeout of an earlier step; synchronizes nothing. */
+yaspmv_status yaspmv_comm_check(yaspmv_comm c);
+int32_t yaspmv_launches_per_fused_step(yaspmv_matrix A);
+/* NULL-safe; unmaps the peers and frees the allocation (synchronize first; peers must not
+ * write into this comm any more). */
+void yaspmv_comm_free(yaspmv_comm c);
+
 /* ---------------------------------------------------------------- misc */
 const char* yaspmv_last_error(void);
 const char* yaspmv_version(void);

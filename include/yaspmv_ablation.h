@@ -18,7 +18,18 @@ extern "C" {
  *   variant 1 "Efficient segmented sum/scan": matrix-based segmented sum, carries across
  *             workgroups by a second kernel after the first completes;
  *   variant 2 "Adjacent synchronization": carries by look-back, workgroup scan never skipped;
- *   variant 3 "Fine-grain optimizations": = yaspmv_spmv.
+ *   variant 3 "Fine-grain optimizations": = yaspmv_spmv;
+ *   variant 4 roofline probe "stream + gather": K1's tile loads and x gathers exactly as
+ *             issued by yaspmv_spmv, then nothing but a per-thread sum (no segmented sum,
+ *             scan, carries or y stores; y's contents are unspecified) — the time any kernel that
+ *             reads this format and gathers x must spend;
+ *   variant 5 roofline probe "stream only": as 4 with every gather redirected to
+ *             x[col & 15] (L1 hits): the format stream alone;
+ *   variant 6 roofline probe "stream + L2 gather": as 4 with every gather redirected to
+ *             x[col & (2^20 - 1)] (an L2-resident 4-8 MB window: L1 misses, L2 hits) —
+ *             separates the cost of the gather requests from that of x's DRAM misses.
+ *             Needs n >= 2^20.
+ * Variants 4 and 5 do not compute y; they exist to measure.
  * x, y: device; the column storage is whatever A was built with (the caller builds A with
  * col_mode I32 for steps 1-2 and the auto/short mode for step 3). */
 yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream);

@@ -21,12 +21,19 @@ KEEP_HOST, DROP_CSR, GPU_ENCODE, TICKET_IDS, NO_PDL = 1, 2, 4, 8, 16
 ARR = {"flags": 0, "col": 1, "col_delta": 2, "val0": 3, "val1": 4, "val2": 5, "val3": 6,
        "seg_row": 7, "zero_rows": 8, "cta_seg0": 9, "fre": 10}
 
+MAX_RANKS = 8  # YASPMV_MAX_RANKS
+IPC_HANDLE_BYTES = 64
+
 # every symbol include/yaspmv.h declares (checked by tests/test_abi.py)
 EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv", "yaspmv_spmv_host",
             "yaspmv_tune", "yaspmv_reencode", "yaspmv_get_info", "yaspmv_export", "yaspmv_export_device",
             "yaspmv_nrm2sq", "yaspmv_nrm2sq_scratch_bytes", "yaspmv_scale", "yaspmv_last_error",
             "yaspmv_version", "yaspmv_launches_per_spmv", "yaspmv_spmv_host_async", "yaspmv_host_sync",
             "yaspmv_spmv_power", "yaspmv_launches_per_power_step", "yaspmv_tune_ex",
+            "yaspmv_comm_create", "yaspmv_comm_ipc_handle", "yaspmv_comm_open_ipc", "yaspmv_comm_connect_local",
+            "yaspmv_comm_x", "yaspmv_comm_begin", "yaspmv_power_step_fused", "yaspmv_comm_wait",
+            "yaspmv_comm_norm2_device", "yaspmv_comm_seq", "yaspmv_comm_check", "yaspmv_launches_per_fused_step",
+            "yaspmv_comm_free",
             # include/yaspmv_ablation.h
             "yaspmv_ablation_spmv", "yaspmv_ablation_tree", "yaspmv_ablation_tree_scratch_bytes"]
 
@@ -99,6 +106,19 @@ def _load():
         "yaspmv_host_sync": ([H], ctypes.c_int),
         "yaspmv_spmv_power": ([H, vp, vp, vp, vp, vp], ctypes.c_int),
         "yaspmv_launches_per_power_step": ([H], i32),
+        "yaspmv_comm_create": ([i32, i32, i32, i64, ctypes.c_int, i32, ctypes.POINTER(H)], ctypes.c_int),
+        "yaspmv_comm_ipc_handle": ([H, vp, i64], ctypes.c_int),
+        "yaspmv_comm_open_ipc": ([H, vp, i64], ctypes.c_int),
+        "yaspmv_comm_connect_local": ([H, ctypes.POINTER(H), i32], ctypes.c_int),
+        "yaspmv_comm_x": ([H, i32], vp),
+        "yaspmv_comm_begin": ([H], ctypes.c_int),
+        "yaspmv_power_step_fused": ([H, H, vp], ctypes.c_int),
+        "yaspmv_comm_wait": ([H, vp], ctypes.c_int),
+        "yaspmv_comm_norm2_device": ([H], vp),
+        "yaspmv_comm_seq": ([H], i64),
+        "yaspmv_comm_check": ([H], ctypes.c_int),
+        "yaspmv_launches_per_fused_step": ([H], i32),
+        "yaspmv_comm_free": ([H], None),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

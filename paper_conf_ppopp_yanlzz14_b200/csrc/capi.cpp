@@ -308,7 +308,7 @@ int64_t alg_bytes(const yaspmv_matrix A) {
 }
 
 yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2 = nullptr,
-                       double* out_norm2 = nullptr, int ablate = 0) {
+                       double* out_norm2 = nullptr, int ablate = 0, const PeerOut* peers = nullptr) {
   const Canonical& c = A->can;
   const Params& p = c.p;
   cudaStream_t cs = (cudaStream_t)stream;
@@ -317,7 +317,10 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
     return YASPMV_OK;
   }
   if (c.ntiles == 0) {
-    CUDA_TRY(cudaMemsetAsync(y, 0, (size_t)c.m * A->vsize, cs));
+    if (peers)
+      for (int q = 0; q < peers->n; ++q) CUDA_TRY(cudaMemsetAsync(peers->p[q], 0, (size_t)c.m * A->vsize, cs));
+    else
+      CUDA_TRY(cudaMemsetAsync(y, 0, (size_t)c.m * A->vsize, cs));
     if (out_norm2) CUDA_TRY(cudaMemsetAsync(out_norm2, 0, sizeof(double), cs));
     return YASPMV_OK;
   }
@@ -358,6 +361,12 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   a.block_ids = (p.flags & YASPMV_TICKET_IDS) ? 0 : 1;
   a.pdl = (p.flags & YASPMV_NO_PDL) ? 0 : 1;
   a.dep_row = nullptr;
+  a.npeer = 0;
+  for (int q = 0; q < YASPMV_MAX_RANKS; ++q) a.peer_out[q] = nullptr;
+  if (peers && p.S == 1) {  // S > 1: the kernel writes tmp, the combine writes the peers
+    a.npeer = peers->n;
+    for (int q = 0; q < peers->n; ++q) a.peer_out[q] = peers->p[q];
+  }
   if (ablate & ABL_DEFER_CARRY) {
     if (p.h != 1 || p.S != 1) return fail(YASPMV_EUNSUPPORTED, "ablation variants need h = 1, S = 1");
     if (A->abl_ntiles < c.ntiles) {
@@ -369,6 +378,7 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
     a.dep_row = A->d_dep_row;
   }
   if (p.S == 1) a.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
+  if (a.npeer > 0 && a.epi == 0) a.epi = 4;  // peer stores live in the EPI instances only
   A->kern->launch(a, p.C, A->grid, stream);
   CUDA_TRY(cudaGetLastError());
   if (ablate & ABL_DEFER_CARRY) {
@@ -376,7 +386,8 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
     CUDA_TRY(cudaGetLastError());
   }
   if (p.S > 1) {
-    launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream, in_norm2, out_norm2 ? A->d_part : nullptr);
+    launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream, in_norm2, out_norm2 ? A->d_part : nullptr,
+                   peers);
     CUDA_TRY(cudaGetLastError());
   }
   if (out_norm2) {
@@ -390,6 +401,11 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
 
 yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags) {
   return install_canonical_impl(A, std::move(c), flags);
+}
+
+yaspmv_status run_spmv_peers(yaspmv_matrix A, const void* x, const double* in_norm2, double* out_norm2,
+                             const yaspmv::PeerOut& peers, void* stream) {
+  return run_spmv(A, x, nullptr, stream, in_norm2, out_norm2, 0, &peers);
 }
 
 // =====================================================================================
@@ -548,8 +564,13 @@ int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
 yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle");
-  if (variant < 1 || variant > 3) return fail(YASPMV_EINVAL, "ablation variant must be 1, 2 or 3");
-  const int ab = variant == 1 ? ABL_DEFER_CARRY : variant == 2 ? ABL_NO_SKIP : 0;
+  if (variant < 1 || variant > 6) return fail(YASPMV_EINVAL, "ablation variant must be in 1..6");
+  const int ab = variant == 1   ? ABL_DEFER_CARRY
+                 : variant == 2 ? ABL_NO_SKIP
+                 : variant == 4 ? ABL_GATHER_ONLY
+                 : variant == 5 ? ABL_STREAM_ONLY
+                 : variant == 6 ? (ABL_GATHER_ONLY | ABL_GATHER_L2)
+                                : 0;
   return run_spmv(A, x, y, stream, nullptr, nullptr, ab);
 }
 

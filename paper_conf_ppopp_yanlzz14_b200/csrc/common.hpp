@@ -13,7 +13,16 @@ namespace yaspmv {
 enum ColMode { COL_U16 = 1, COL_I32 = 2, COL_DELTA = 3 };
 enum EmptyMode { EMPTY_FILLER = 1, EMPTY_MAP = 2 };
 // ablation switches (Fig. 14); never set by yaspmv_spmv
-enum Ablate { ABL_DEFER_CARRY = 1, ABL_NO_SKIP = 2 };
+enum Ablate {
+  ABL_DEFER_CARRY = 1,
+  ABL_NO_SKIP = 2,
+  // roofline probes (not steps of the method): the tile's loads exactly as K1 issues them,
+  // then only a per-thread sum kept live; GATHER_ONLY keeps the x gathers, STREAM_ONLY
+  // redirects them to x[col & 15] (L1 hits) so only the format stream remains
+  ABL_GATHER_ONLY = 4,
+  ABL_STREAM_ONLY = 8,
+  ABL_GATHER_L2 = 16  // with GATHER_ONLY: gathers of x[col & (2^20-1)] (4-8 MB: L2 hits, L1 misses)
+};
 
 struct Params {
   int h = 1, w = 1, S = 1, T = 16, C = 256, col_mode = 0, empty_mode = 0, flags = 0;
@@ -123,6 +132,17 @@ struct KArgs {
   int block_ids;           // 1: tile = blockIdx (in-order dispatch), ticket only for the epoch
   int pdl;                 // launched with programmatic dependent launch
   int64_t* dep_row;        // ABL_DEFER_CARRY: per tile, row of the carried segment or -1
+  // fused exchange (yaspmv_power_step_fused, EPI instances only): npeer > 0 writes every
+  // output element to peer_out[q][i] for q < npeer (every rank's copy of the next x,
+  // pre-offset to this rank's chunk) instead of out[i]
+  int npeer;
+  void* peer_out[YASPMV_MAX_RANKS];
+};
+
+// destinations of a fused exchange (combine kernel of BCCOO+, S > 1)
+struct PeerOut {
+  int n = 0;
+  void* p[YASPMV_MAX_RANKS] = {};
 };
 
 typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
@@ -138,7 +158,7 @@ const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm);
 const std::vector<KernelEntry>& all_kernels();
 
 void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream,
-                    const double* in_norm2 = nullptr, double* part = nullptr);
+                    const double* in_norm2 = nullptr, double* part = nullptr, const PeerOut* peers = nullptr);
 int64_t combine_blocks(int64_t m);
 void launch_sum_f64(const double* v, int64_t n, double* out, double* partials, void* stream);
 void launch_carry_fixup(const unsigned long long* status, const double* carry, const int64_t* dep_row,

@@ -88,3 +88,7 @@ struct yaspmv_matrix_s {
 
 // capi.cpp: make an already encoded Canonical the handle's encoding (kernel + upload)
 yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags);
+// capi.cpp: one power-iteration SpMV whose output goes to peers.p[q] (q < peers.n) instead
+// of a local y (the fused exchange of comm.cu); out_norm2 receives sum y^2 (nullable)
+yaspmv_status run_spmv_peers(yaspmv_matrix A, const void* x, const double* in_norm2, double* out_norm2,
+                             const yaspmv::PeerOut& peers, void* stream);

@@ -16,7 +16,7 @@ __device__ __forceinline__ double block_sum256(double v);
 // optional power-iteration epilogue: y scaled by 1/sqrt(*in_norm2), block partials of y^2
 template <typename VT>
 __global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, int64_t m, int64_t stride, int S,
-                               const double* __restrict__ in_norm2, double* __restrict__ part) {
+                               const double* __restrict__ in_norm2, double* __restrict__ part, const PeerOut peers) {
   cudaTriggerProgrammaticLaunchCompletion();
   const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
   const double inv = in_norm2 ? 1.0 / sqrt(in_norm2[0]) : 1.0;
@@ -25,7 +25,13 @@ __global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, i
     double s = (double)__ldcs(tmp + i);
     for (int q = 1; q < S; ++q) s += (double)__ldcs(tmp + (int64_t)q * stride + i);
     const VT o = in_norm2 ? (VT)((VT)s * inv) : (VT)s;
-    y[i] = o;
+    if (peers.n > 0) {  // fused exchange: every rank's copy of the next x (yaspmv_power_step_fused)
+#pragma unroll
+      for (int q = 0; q < YASPMV_MAX_RANKS; ++q)
+        if (q < peers.n) static_cast<VT*>(peers.p[q])[i] = o;
+    } else {
+      y[i] = o;
+    }
     ss += (double)o * (double)o;
   }
   if (part) {
@@ -53,15 +59,16 @@ int64_t combine_blocks(int64_t m) {
 }
 
 void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream,
-                    const double* in_norm2, double* part) {
+                    const double* in_norm2, double* part, const PeerOut* peers) {
   if (m <= 0) return;
   const int64_t blocks = combine_blocks(m);
+  const PeerOut po = peers ? *peers : PeerOut();
   if (dtype == 0)
     combine_kernel<float><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const float*)tmp, (float*)y, m,
-                                                                             stride, S, in_norm2, part);
+                                                                             stride, S, in_norm2, part, po);
   else
     combine_kernel<double><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const double*)tmp, (double*)y, m,
-                                                                               stride, S, in_norm2, part);
+                                                                               stride, S, in_norm2, part, po);
 }
 
 // ---------------------------------------------------------------- ||v||^2

@@ -171,6 +171,22 @@ __device__ __forceinline__ double ld_relaxed_f64(const double* p) {
 }
 }  // namespace dev
 
+// Output store.  In a fused exchange (EPI instances with npeer > 0) the element goes to
+// every rank's copy of the next x over peer memory (NVLink P2P stores through IPC
+// mappings; the rank's own buffer is one of them), so the all-gather overlaps the SpMV.
+template <typename VT, bool EPI>
+__device__ __forceinline__ void store_out(const KArgs& a, VT* out, int64_t i, VT v) {
+  if constexpr (EPI) {
+    if (a.npeer > 0) {
+#pragma unroll
+      for (int q = 0; q < YASPMV_MAX_RANKS; ++q)
+        if (q < a.npeer) static_cast<VT*>(a.peer_out[q])[i] = v;
+      return;
+    }
+  }
+  out[i] = v;
+}
+
 template <typename VT, int H, int W, int T, int CM>
 struct KTraits {
   static constexpr int VB = T * W * (int)sizeof(VT);      // value bytes per thread per array
@@ -232,7 +248,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
       const int64_t sr = a.zero_rows[z];
 #pragma unroll
       for (int r = 0; r < H; ++r)
-        if (sr * H + r < a.out_limit) out[sr * H + r] = VT(0);
+        if (sr * H + r < a.out_limit) store_out<VT, EPI>(a, out, sr * H + r, VT(0));
     }
   }
   // row stops: '0' bits; one popc gives their count
@@ -259,7 +275,12 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   const VT* x = static_cast<const VT*>(a.x);
   VT xs[T][W];
 #pragma unroll
-  for (int b = 0; b < T; ++b) dev::gather_x<VT, W>(x, colb[b], a.n, pol_x, xs[b]);
+  for (int b = 0; b < T; ++b)
+    dev::gather_x<VT, W>(x,
+                         (a.ablate & (ABL_STREAM_ONLY | ABL_GATHER_L2))
+                             ? (colb[b] & ((a.ablate & ABL_STREAM_ONLY) ? 15 : 0xFFFFF))
+                             : colb[b],
+                         a.n, pol_x, xs[b]);
 
   // ---- step 2a: multiply + per-thread sequential segmented sum ------
   // Strategy 1: the per-block products stay in registers ("intermediate_sums",
@@ -280,6 +301,16 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
       pr[b][r] = p;
       acc[r] = stop ? VT(0) : acc[r] + p;
     }
+  }
+
+  if (a.ablate & (ABL_GATHER_ONLY | ABL_STREAM_ONLY)) {  // roofline probes: loads only
+    VT s = VT(0);
+#pragma unroll
+    for (int b = 0; b < T; ++b)
+#pragma unroll
+      for (int r = 0; r < H; ++r) s += pr[b][r];
+    if (s == VT(-1.25e-30) || fl == 0x9e3779b9u) out[t] = s;  // keeps every load live
+    return;
   }
 
   // ---- step 2b: CTA segmented scan of (has_stop, last partial sum) --
@@ -383,12 +414,11 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
             for (int r = 0; r < H; ++r) dep[r] = run[r];
             dep_row = row;
           } else {
-            VT* op = out + row * H;
 #pragma unroll
             for (int r = 0; r < H; ++r)
               if (H == 1 || row * H + r < a.out_limit) {
                 const VT o = EPI ? run[r] * invv : run[r];
-                op[r] = o;
+                store_out<VT, EPI>(a, out, row * H + r, o);
                 if constexpr (EPI) ssv = fma(o, o, ssv);
               }
           }
@@ -415,7 +445,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
             for (int r = 0; r < H; ++r)
               if (sr * H + r < a.out_limit) {
                 const VT o = EPI ? run[r] * invv : run[r];
-                out[sr * H + r] = o;
+                store_out<VT, EPI>(a, out, sr * H + r, o);
                 if constexpr (EPI) ssv = fma(o, o, ssv);
               }
           }
@@ -483,7 +513,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
     for (int r = 0; r < H; ++r)
       if (dep_row * H + r < a.out_limit) {
         const VT o = (VT)(((double)dep[r] + carry[r]) * inv);
-        out[dep_row * H + r] = o;
+        store_out<VT, EPI>(a, out, dep_row * H + r, o);
         ds += (double)o * (double)o;
       }
     if (EPI && (a.epi & 2)) a.part[tile * (NW + 1) + NW] = ds;

@@ -166,3 +166,76 @@ class PowerIteration:
         if self.fused and not self.first:
             return self.x / self.norm_prev.sqrt().to(self.x.dtype)
         return self.x
+
+
+class FusedPowerIteration:
+    """The power iteration with the exchange fused into the SpMV (yaspmv_power_step_fused,
+    SURVEY.md §8(f) NEXT #1): each rank's SpMV stores its rows of z_k directly into every
+    rank's copy of the next x over peer memory (NVLink P2P through CUDA IPC), and a one-warp
+    publish / wait kernel pair replaces the NCCL all-reduce + all-gather.  One call of
+    ``step`` = wait for the peers' previous step + SpMV (+ BCCOO+ combine) + ||z||^2 + publish,
+    all on the device; the host never blocks.
+
+    ``comm``: an already connected ``Comm`` (tests: several ranks as several handles of one
+    process, ``Comm.connect_local``); otherwise one is created on ``device`` and, for
+    world > 1, the ranks exchange IPC handles over ``group`` (torch.distributed
+    all_gather_object) and map each other's buffers.  ``comm_factory`` replaces the Comm
+    class (CPU tests of the exchange logic)."""
+
+    def __init__(self, layout: Layout, A, dtype, device, group=None, comm=None, timeout_ms: int = 0,
+                 comm_factory=None):
+        import torch
+        self.L = layout
+        self.A = A
+        self.group = group
+        self.device = torch.device(device)
+        self.own_comm = comm is None
+        if comm is None:
+            if comm_factory is None:
+                from .matrix import Comm as comm_factory
+            npdt = np.float32 if dtype == torch.float32 else np.float64
+            comm = comm_factory(self.device.index or 0, layout.rank, layout.world, layout.m_max, npdt, timeout_ms)
+            if layout.world > 1:
+                import torch.distributed as dist
+                handles = [None] * layout.world
+                dist.all_gather_object(handles, comm.ipc_handle(), group=group)
+                comm.open_ipc(handles)
+        self.comm = comm
+        self.restart()
+
+    def restart(self):
+        """x_0 = 1/sqrt(N) on the real entries of this rank's copy, then (world > 1, own comm)
+        a barrier so that no peer writes into a buffer before every rank is ready."""
+        import torch
+        L = self.L
+        x = self.comm.x(0)
+        x.zero_()
+        n_true = int(L.bounds[-1])
+        for r in range(L.world):
+            a = r * L.m_max
+            x[a: a + int(L.bounds[r + 1] - L.bounds[r])] = 1.0 / np.sqrt(max(n_true, 1))
+        self.comm.begin()
+        if self.own_comm and L.world > 1:
+            import torch.distributed as dist
+            if self.device.type == "cuda":
+                torch.cuda.synchronize(self.device)
+            dist.barrier(group=self.group)
+        self.first = True
+
+    def step(self, stream=None):
+        self.A.power_step_fused(self.comm, stream)
+        self.first = False
+
+    def launches_per_step(self) -> int:
+        return self.A.launches_per_fused_step()
+
+    def z(self):
+        """The latest unnormalised iterate z_k (this rank's replicated copy, padded layout)."""
+        return self.comm.x(0)
+
+    def current_x(self, stream=None):
+        """x_k = z_k / ||z_k|| (materialised; waits on the device for every peer's step)."""
+        if self.first:
+            return self.comm.x(0).clone()
+        self.comm.wait(stream)
+        return self.comm.x(0) / self.comm.norm2().sqrt().to(self.comm.x(0).dtype)

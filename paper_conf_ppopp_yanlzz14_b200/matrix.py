@@ -115,6 +115,14 @@ class Matrix:
     def launches_per_power_step(self) -> int:
         return int(lib.yaspmv_launches_per_power_step(self._h))
 
+    def power_step_fused(self, comm: "Comm", stream=None) -> None:
+        """One fused power step over `comm` (yaspmv_power_step_fused): z_k of this rank's
+        rows goes straight into every rank's copy of the next x."""
+        check(lib.yaspmv_power_step_fused(self._h, comm._h, _stream(stream)))
+
+    def launches_per_fused_step(self) -> int:
+        return int(lib.yaspmv_launches_per_fused_step(self._h))
+
     def spmv_host(self, x: np.ndarray, y: np.ndarray | None = None, stream=None) -> np.ndarray:
         """y := A·x with host arrays (copies in and out inside the call)."""
         x = np.ascontiguousarray(x, dtype=self.dtype)
@@ -168,6 +176,82 @@ class Matrix:
         out = np.empty(nb.value, dtype=np.uint8)
         check(fn(self._h, _lib.ARR[name], out.ctypes.data if nb.value else None, nb.value, ctypes.byref(nb)))
         return out.view(self._arr_dtype(name))
+
+
+class Comm:
+    """The replicated x of a row-partitioned power iteration (yaspmv_comm, include/yaspmv.h
+    "fused multi-GPU power step"): two x buffers + a signal pad in one device allocation,
+    mapped by every peer."""
+
+    def __init__(self, device: int, rank: int, world: int, chunk: int, dtype, timeout_ms: int = 0):
+        self.dtype = np.dtype(dtype)
+        self.device, self.rank, self.world, self.chunk = device, rank, world, chunk
+        h = ctypes.c_void_p()
+        check(lib.yaspmv_comm_create(device, rank, world, chunk, _DT[self.dtype], timeout_ms, ctypes.byref(h)))
+        self._h = h
+
+    def ipc_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(_lib.IPC_HANDLE_BYTES)
+        check(lib.yaspmv_comm_ipc_handle(self._h, buf, _lib.IPC_HANDLE_BYTES))
+        return buf.raw
+
+    def open_ipc(self, handles: list[bytes]) -> None:
+        blob = b"".join(h if h is not None else bytes(_lib.IPC_HANDLE_BYTES) for h in handles)
+        check(lib.yaspmv_comm_open_ipc(self._h, blob, len(blob)))
+
+    def connect_local(self, peers: list["Comm"]) -> None:
+        arr = (ctypes.c_void_p * len(peers))(*[p._h.value for p in peers])
+        check(lib.yaspmv_comm_connect_local(self._h, arr, len(peers)))
+
+    def x(self, which: int = 0):
+        """torch view of x buffer (seq + which) % 2 (which = 0: the next step's input /
+        the latest z; 1: the buffer the next step writes), world * chunk elements."""
+        import torch
+        ptr = lib.yaspmv_comm_x(self._h, which)
+        n = self.world * self.chunk
+        tdt = torch.float32 if self.dtype == np.float32 else torch.float64
+        return _device_view(ptr, n, tdt, self.device)
+
+    def norm2(self):
+        """torch view of the device double written by wait(): total ||z||^2."""
+        import torch
+        return _device_view(lib.yaspmv_comm_norm2_device(self._h), 1, torch.float64, self.device)
+
+    def begin(self) -> None:
+        check(lib.yaspmv_comm_begin(self._h))
+
+    def wait(self, stream=None) -> None:
+        check(lib.yaspmv_comm_wait(self._h, _stream(stream)))
+
+    def check(self) -> None:
+        check(lib.yaspmv_comm_check(self._h))
+
+    @property
+    def seq(self) -> int:
+        return int(lib.yaspmv_comm_seq(self._h))
+
+    def free(self) -> None:
+        if self._h is not None and self._h.value:
+            lib.yaspmv_comm_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def _device_view(ptr: int, n: int, tdt, device: int):
+    """A torch tensor over n elements of raw device memory owned by libyaspmv (no copy)."""
+    import torch
+    itemsize = torch.empty(0, dtype=tdt).element_size()
+
+    class _Arr:  # __cuda_array_interface__ shim
+        __cuda_array_interface__ = {"shape": (n,), "typestr": ("<f%d" % itemsize), "data": (ptr, False),
+                                    "version": 3, "strides": None}
+    with torch.cuda.device(device):
+        return torch.as_tensor(_Arr(), device=f"cuda:{device}")
 
 
 def nrm2sq(v, out, scratch, stream=None) -> None:

@@ -118,3 +118,127 @@ def test_power_iteration_world2_matches_single_process(world, fused):
         y, _ = ref.spmv(a.row_ptr, a.col, a.val.astype(np.float64), x, with_bound=False)
         x = y / np.linalg.norm(y)
     assert np.allclose(x_dist, x, rtol=1e-4, atol=1e-6)
+
+
+# ---------------------------------------------------------------- fused exchange (host side)
+class _ShmComm:
+    """CPU model of yaspmv_comm for the host logic of dist.FusedPowerIteration on gloo:
+    the "device allocation" is a shared file ([x0 | x1 | flags | norms[2][P]], fp64 here),
+    the "IPC handle" its path; the protocol (parity, epochs, rank-order norm sum) mirrors
+    csrc/comm.cu."""
+
+    def __init__(self, device, rank, world, chunk, dtype, timeout_ms, root=None):
+        self.rank, self.world, self.chunk = rank, world, chunk
+        self.n = world * chunk
+        self.path = os.path.join(root or os.environ["SHM_ROOT"], f"comm{rank}")
+        self.size = 2 * self.n + 3 * world
+        self.buf = torch.from_file(self.path, shared=True, size=self.size, dtype=torch.float64)
+        self.buf.zero_()
+        self.peers = None
+        self.seq, self.fresh = 0, True
+        self.total = torch.zeros(1, dtype=torch.float64)
+
+    def _x(self, b, k):
+        return b[(k % 2) * self.n: (k % 2 + 1) * self.n]
+
+    def _flags(self, b):
+        return b[2 * self.n: 2 * self.n + self.world]
+
+    def _norms(self, b, parity):
+        o = 2 * self.n + self.world + parity * self.world
+        return b[o: o + self.world]
+
+    def ipc_handle(self):
+        return self.path.encode()
+
+    def open_ipc(self, handles):
+        assert len(handles) == self.world and handles[self.rank] == self.path.encode()
+        self.peers = [torch.from_file(h.decode(), shared=True, size=self.size, dtype=torch.float64)
+                      for h in handles]
+
+    def x(self, which=0):
+        return self._x(self.buf, self.seq + which)
+
+    def norm2(self):
+        return self.total
+
+    def begin(self):
+        self.fresh = True
+
+    def wait(self, stream=None):
+        import time
+        t0 = time.time()
+        while float(self._flags(self.buf).min()) < self.seq:
+            assert time.time() - t0 < 60, "peer never published"
+            time.sleep(0.001)
+        self.total[0] = float(sum(float(v) for v in self._norms(self.buf, (self.seq - 1) % 2)))
+
+    def check(self):
+        pass
+
+
+class _ShmFusedMatrix:
+    """The rank's rows on the CPU (oracle product) behind the fused-step interface."""
+
+    def __init__(self, csr, m_local):
+        self.csr, self.m = csr, m_local
+
+    def power_step_fused(self, c, stream=None):
+        if not c.fresh:
+            c.wait()
+        x = c._x(c.buf, c.seq).numpy()
+        z, _ = ref.spmv(self.csr.row_ptr, self.csr.col, self.csr.val, x, with_bound=False)
+        if not c.fresh:
+            z = z / np.sqrt(float(c.total[0]))
+        n2 = float(np.sum(z ** 2))
+        for p in c.peers:  # peer stores, then norm + flag (the publish kernel)
+            c._x(p, c.seq + 1)[c.rank * c.chunk: c.rank * c.chunk + self.m] = torch.from_numpy(z)
+            c._norms(p, c.seq % 2)[c.rank] = n2
+            c._flags(p)[c.rank] = c.seq + 1
+        c.seq += 1
+        c.fresh = False
+
+    def launches_per_fused_step(self):
+        return 0
+
+
+def _fused_worker(rank, world, port, root, n, iters):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ["SHM_ROOT"] = root
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    kw = dict(n=n, n_net=2, net_log2=(8, 10), band=512)
+    from synth import matrices as sm
+    full = sm.circuit_like_rows(0, n, **kw)
+    L = D.make_layout(full.row_ptr, rank, world)
+    sub = full.row_slice(L.r0, L.r1)
+    sub.col = D.remap_columns(sub.col, L.bounds, L.m_max)
+    sub.val = sub.val.astype(np.float64)
+    pit = D.FusedPowerIteration(L, _ShmFusedMatrix(sub, L.m_local), torch.float64, "cpu",
+                                comm_factory=_ShmComm)
+    for _ in range(iters):
+        pit.step()
+    x = pit.current_x()
+    np.save(os.path.join(root, f"x{rank}.npy"), D.unpad(x.numpy(), L.bounds, L.m_max))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_fused_power_iteration_host_protocol_world2():
+    """dist.FusedPowerIteration over gloo world 2: IPC-handle exchange in rank order, x_0
+    layout, restart barrier, and the parity/epoch protocol of comm.cu (modelled on shared
+    files) give every rank the single-process power iteration."""
+    import torch.multiprocessing as mp
+    n, iters, world = 1 << 12, 4, 2
+    with tempfile.TemporaryDirectory() as td:
+        mp.spawn(_fused_worker, args=(world, _free_port(), td, n, iters), nprocs=world, join=True)
+        xs = [np.load(os.path.join(td, f"x{r}.npy")) for r in range(world)]
+    from synth import matrices as sm
+    a = sm.circuit_like_rows(0, n, n=n, n_net=2, net_log2=(8, 10), band=512)
+    x = np.full(n, 1.0 / np.sqrt(n))
+    for _ in range(iters):
+        y, _ = ref.spmv(a.row_ptr, a.col, a.val.astype(np.float64), x, with_bound=False)
+        x = y / np.linalg.norm(y)
+    for xr in xs:
+        assert np.allclose(xr, x, rtol=1e-12, atol=1e-15)
