@@ -56,9 +56,12 @@ enum {
                             workgroup id, relying on in-order dispatch as the paper does
                             ("Current GPUs dispatch workgroups in-order"); the
                             ticket then only yields the launch epoch                       */
-  YASPMV_NO_PDL = 16     /* launch without programmatic dependent launch (by default each
+  YASPMV_NO_PDL = 16,    /* launch without programmatic dependent launch (by default each
                             SpMV may start streaming its matrix tiles while the previous
                             kernel on the stream drains; x, y and carries wait for it)     */
+  YASPMV_FORCE_HANDOFF = 32 /* testing: a tile always hands its carried first segment to the
+                            predecessor hand-off protocol, even when the predecessor's
+                            carry is already published (results are identical)            */
 };
 
 /* Tunable parameters, Table 1.  0 in any field = auto/default. */

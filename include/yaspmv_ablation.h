@@ -28,7 +28,13 @@ extern "C" {
  *   variant 6 roofline probe "stream + L2 gather": as 4 with every gather redirected to
  *             x[col & (2^20 - 1)] (an L2-resident 4-8 MB window: L1 misses, L2 hits) —
  *             separates the cost of the gather requests from that of x's DRAM misses.
- *             Needs n >= 2^20.
+ *             Needs n >= 2^20;
+ *   variant 7 roofline probe "no carries": variant 1 without its carry kernel — every
+ *             segment that spans a workgroup boundary is left without its carry-in (y wrong
+ *             there): the cost of adjacent synchronization is the difference to variant 3;
+ *   variant 8 roofline probe "up to the scan": returns after the workgroup segmented scan
+ *             (no carry publish, no y stores, no look-back);
+ *   variant 9 roofline probe: variant 7 without the y stores of the write-back.
  * Variants 4 and 5 do not compute y; they exist to measure.
  * x, y: device; the column storage is whatever A was built with (the caller builds A with
  * col_mode I32 for steps 1-2 and the auto/short mode for step 3). */

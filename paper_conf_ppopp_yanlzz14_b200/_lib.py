@@ -17,7 +17,7 @@ OK, EINVAL, ENOMEM, ECUDA, EUNSUPPORTED = 0, 1, 2, 3, 4
 F32, F64 = 0, 1
 COL_AUTO, COL_U16, COL_I32, COL_DELTA16 = 0, 1, 2, 3
 EMPTY_AUTO, EMPTY_FILLER, EMPTY_MAP = 0, 1, 2
-KEEP_HOST, DROP_CSR, GPU_ENCODE, TICKET_IDS, NO_PDL = 1, 2, 4, 8, 16
+KEEP_HOST, DROP_CSR, GPU_ENCODE, TICKET_IDS, NO_PDL, FORCE_HANDOFF = 1, 2, 4, 8, 16, 32
 ARR = {"flags": 0, "col": 1, "col_delta": 2, "val0": 3, "val1": 4, "val2": 5, "val3": 6,
        "seg_row": 7, "zero_rows": 8, "cta_seg0": 9, "fre": 10}
 

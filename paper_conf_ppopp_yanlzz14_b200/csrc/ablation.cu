@@ -15,29 +15,31 @@ namespace yaspmv {
 // of the published values back to the nearest tile holding a segment end (state 2),
 // folded newest to oldest (fixed order, deterministic).  Runs after all tiles published.
 template <typename VT>
-__global__ void carry_fixup_kernel(const unsigned long long* status, const double* carry, const int64_t* dep_row,
-                                   int64_t ntiles, VT* y) {
+__global__ void carry_fixup_kernel(const unsigned long long* status, int sstride, const double* carry,
+                                   const int64_t* dep_row, int64_t ntiles, VT* y) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < ntiles; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = dep_row[k];
     if (r < 0) continue;
     double c = 0.0;
     for (int64_t i = k - 1; i >= 0; --i) {
       c += carry[i];
-      if ((status[i] & 3ull) == 2ull) break;
+      if ((status[i * sstride] & 3ull) == 2ull) break;
     }
     y[r] = (VT)((double)y[r] + c);
   }
 }
 
 void launch_carry_fixup(const unsigned long long* status, const double* carry, const int64_t* dep_row,
-                        int64_t ntiles, void* y, int dtype, void* stream) {
+                        int64_t ntiles, void* y, int dtype, void* stream, int sstride) {
   int64_t g = (ntiles + 255) / 256;
   if (g < 1) g = 1;
   if (g > 65535) g = 65535;
   if (dtype == 0)
-    carry_fixup_kernel<float><<<(unsigned)g, 256, 0, (cudaStream_t)stream>>>(status, carry, dep_row, ntiles, (float*)y);
+    carry_fixup_kernel<float><<<(unsigned)g, 256, 0, (cudaStream_t)stream>>>(status, sstride, carry, dep_row, ntiles,
+                                                                               (float*)y);
   else
-    carry_fixup_kernel<double><<<(unsigned)g, 256, 0, (cudaStream_t)stream>>>(status, carry, dep_row, ntiles, (double*)y);
+    carry_fixup_kernel<double><<<(unsigned)g, 256, 0, (cudaStream_t)stream>>>(status, sstride, carry, dep_row, ntiles,
+                                                                                (double*)y);
 }
 
 // Tree-based segmented sum over 1024-element tiles (256 threads x 4 elements): products

@@ -103,9 +103,13 @@ yaspmv_status alloc_scratch(const Canonical& c, int vsize, DevArrays& d) {
   CUDA_TRY(cudaMalloc((void**)&d.ticket, sizeof(unsigned long long)));
   CUDA_TRY(cudaMemset(d.ticket, 0, sizeof(unsigned long long)));
   const int64_t nt = std::max<int64_t>(c.ntiles, 1);
-  CUDA_TRY(cudaMalloc((void**)&d.status, nt * sizeof(unsigned long long)));
-  CUDA_TRY(cudaMemset(d.status, 0, nt * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMalloc((void**)&d.status, 2 * nt * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMemset(d.status, 0, 2 * nt * sizeof(unsigned long long)));
   CUDA_TRY(cudaMalloc((void**)&d.carry, nt * p.h * sizeof(double)));
+  CUDA_TRY(cudaMalloc((void**)&d.bnd, 2 * (nt + 1) * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMemset(d.bnd, 0, 2 * (nt + 1) * sizeof(unsigned long long)));
+  CUDA_TRY(cudaMalloc((void**)&d.pend_val, nt * p.h * sizeof(double)));
+  CUDA_TRY(cudaMalloc((void**)&d.pend_row, nt * sizeof(long long)));
   if (p.S > 1) CUDA_TRY(cudaMalloc(&d.tmp, (size_t)p.S * c.MB * p.h * vsize));
   return YASPMV_OK;
 }
@@ -292,7 +296,7 @@ int64_t format_bytes(const yaspmv_matrix A) {
   b += c.nnzb_pad * (int64_t)col_bytes(p.col_mode);             // col / delta
   b += A->n_escapes * 4;                                         // escape reads
   b += c.nnzb_pad / 8;                                           // bit flags
-  b += c.ntiles * (4 + 8 + 8 * (int64_t)p.h);                    // cta_seg0, status, carry
+  b += c.ntiles * (4 + 16 + (p.h > 1 ? 8 * (int64_t)p.h : 0) + 16);  // cta_seg0, status(+carry), carries, hand-off
   if (c.has_seg_row) b += c.n_stops * 4;                         // seg_row
   b += c.n_zero * 4;                                             // zero-fill list
   return b;
@@ -354,6 +358,10 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   a.ticket = A->d.ticket;
   a.status = A->d.status;
   a.carry = A->d.carry;
+  a.bnd = A->d.bnd;
+  a.pend_val = A->d.pend_val;
+  a.pend_row = A->d.pend_row;
+  a.force_handoff = (p.flags & YASPMV_FORCE_HANDOFF) ? 1 : 0;
   a.epi = 0;
   a.in_norm2 = in_norm2;
   a.part = A->d_part;
@@ -375,14 +383,14 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
       CUDA_TRY(cudaMalloc((void**)&A->d_dep_row, c.ntiles * sizeof(int64_t)));
       A->abl_ntiles = c.ntiles;
     }
-    a.dep_row = A->d_dep_row;
+    a.dep_row = (ablate & ABL_NO_FIXUP) ? nullptr : A->d_dep_row;
   }
   if (p.S == 1) a.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
-  if (a.npeer > 0 && a.epi == 0) a.epi = 4;  // peer stores live in the EPI instances only
+  // (npeer > 0 selects the EPI = 2 instance: epilogue + peer stores)
   A->kern->launch(a, p.C, A->grid, stream);
   CUDA_TRY(cudaGetLastError());
-  if (ablate & ABL_DEFER_CARRY) {
-    launch_carry_fixup(A->d.status, A->d.carry, A->d_dep_row, c.ntiles, y, A->dtype, stream);
+  if ((ablate & ABL_DEFER_CARRY) && !(ablate & ABL_NO_FIXUP)) {
+    launch_carry_fixup(A->d.status, A->d.carry, A->d_dep_row, c.ntiles, y, A->dtype, stream, 2);
     CUDA_TRY(cudaGetLastError());
   }
   if (p.S > 1) {
@@ -564,12 +572,17 @@ int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
 yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle");
-  if (variant < 1 || variant > 6) return fail(YASPMV_EINVAL, "ablation variant must be in 1..6");
+  if (variant < 1 || variant > 9) return fail(YASPMV_EINVAL, "ablation variant must be in 1..9");
+  if (variant != 3 && (A->can.p.h != 1 || A->can.p.w != 1))
+    return fail(YASPMV_EUNSUPPORTED, "ablation variants / probes are compiled for 1x1 blocks only");
   const int ab = variant == 1   ? ABL_DEFER_CARRY
                  : variant == 2 ? ABL_NO_SKIP
                  : variant == 4 ? ABL_GATHER_ONLY
                  : variant == 5 ? ABL_STREAM_ONLY
                  : variant == 6 ? (ABL_GATHER_ONLY | ABL_GATHER_L2)
+                 : variant == 7 ? (ABL_DEFER_CARRY | ABL_NO_FIXUP)
+                 : variant == 8 ? ABL_STOP_SCAN
+                 : variant == 9 ? (ABL_DEFER_CARRY | ABL_NO_FIXUP | ABL_NO_YSTORE)
                                 : 0;
   return run_spmv(A, x, y, stream, nullptr, nullptr, ab);
 }

@@ -21,7 +21,10 @@ enum Ablate {
   // redirects them to x[col & 15] (L1 hits) so only the format stream remains
   ABL_GATHER_ONLY = 4,
   ABL_STREAM_ONLY = 8,
-  ABL_GATHER_L2 = 16  // with GATHER_ONLY: gathers of x[col & (2^20-1)] (4-8 MB: L2 hits, L1 misses)
+  ABL_GATHER_L2 = 16,  // with GATHER_ONLY: gathers of x[col & (2^20-1)] (4-8 MB: L2 hits, L1 misses)
+  ABL_STOP_SCAN = 32,  // probe: return right after the CTA scan (no publish, stores, carries)
+  ABL_NO_FIXUP = 64,  // host side, with DEFER_CARRY: no carry kernel ("no carries" probe)
+  ABL_NO_YSTORE = 256  // probe: y stores of the FILLER write-back skipped
 };
 
 struct Params {
@@ -121,8 +124,20 @@ struct KArgs {
   int64_t ntiles;
   int64_t period;          // tickets per launch = ntiles + grid (persistent CTAs)
   unsigned long long* ticket;
+  // per tile, 16 B: [0] status word (epoch << 2 | state), [1] (h = 1) the carry-out as fp64
+  // bits, written together by one 128-bit store and read by one 128-bit load, so no fence
+  // orders value and status; h > 1 keeps the carries in `carry` (release/relaxed pair)
   unsigned long long* status;
   double* carry;           // ntiles * h
+  // non-blocking carries: bnd[2k..2k+1] is the 16-byte hand-off word between tile k-1 and
+  // tile k (epoch-tagged; whichever of the two arrives second completes tile k's carried
+  // segment).  h = 1: the pending partial and its row travel inside the word (one 128-bit
+  // atomic exchange per side, no fence); h > 1: in pend_val[k*h..] / pend_row[k], ordered
+  // by acquire-release exchanges
+  unsigned long long* bnd;
+  double* pend_val;
+  long long* pend_row;
+  int force_handoff;       // YASPMV_FORCE_HANDOFF (tests): never take the ready-predecessor fast path
   // power-iteration epilogue (yaspmv_spmv_power): bit 0 scale y by 1/sqrt(*in_norm2),
   // bit 1 write per-warp partials of sum y^2 to part[tile*(C/32+1) + warp] (+ carried seg)
   int epi;
@@ -161,8 +176,10 @@ void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, 
                     const double* in_norm2 = nullptr, double* part = nullptr, const PeerOut* peers = nullptr);
 int64_t combine_blocks(int64_t m);
 void launch_sum_f64(const double* v, int64_t n, double* out, double* partials, void* stream);
+// sstride: u64 words per tile in `status` (2 for a matrix's status words, 1 for the tree
+// ablation's scratch)
 void launch_carry_fixup(const unsigned long long* status, const double* carry, const int64_t* dep_row,
-                        int64_t ntiles, void* y, int dtype, void* stream);
+                        int64_t ntiles, void* y, int dtype, void* stream, int sstride = 1);
 int launch_tree_segsum(const int32_t* rows, const uint8_t* flags, const int32_t* tile_seg0, const int32_t* col,
                        const void* val, int64_t n_elem, const void* x, void* y, int64_t m, int dtype,
                        unsigned long long* status, double* carry, int64_t* dep_row, void* stream);

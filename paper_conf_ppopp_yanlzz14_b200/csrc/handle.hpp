@@ -20,10 +20,13 @@ struct DevArrays {
   unsigned long long* ticket = nullptr;
   unsigned long long* status = nullptr;
   double* carry = nullptr;
+  unsigned long long* bnd = nullptr;  // per tile boundary: hand-off word of the carried segment
+  double* pend_val = nullptr;         // per tile: the waiting first segment's partial (h fp64)
+  long long* pend_row = nullptr;      // per tile: its output row
   void* tmp = nullptr;
   void free_all() {
     void* ps[] = {val[0], val[1], val[2], val[3], col, col32, flags, cta_seg0, seg_row, zero_rows,
-                  ticket, status, carry, tmp};
+                  ticket, status, carry, bnd, pend_val, pend_row, tmp};
     for (void* p : ps)
       if (p) cudaFree(p);
     *this = DevArrays();

@@ -164,6 +164,29 @@ __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long lon
   asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ unsigned long long atom_exch_acq_rel(unsigned long long* p, unsigned long long v) {
+  unsigned long long o;
+  asm volatile("atom.acq_rel.gpu.global.exch.b64 %0, [%1], %2;" : "=l"(o) : "l"(p), "l"(v) : "memory");
+  return o;
+}
+// 16-byte status / hand-off words: single 128-bit accesses (LDG/STG.E.128, ATOMG.EXCH.128),
+// so a status word and the value published with it are observed together
+__device__ __forceinline__ void ld_relaxed_16(const unsigned long long* p, unsigned long long& lo,
+                                              unsigned long long& hi) {
+  asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(lo), "=l"(hi) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_16(unsigned long long* p, unsigned long long lo, unsigned long long hi) {
+  asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(lo), "l"(hi) : "memory");
+}
+__device__ __forceinline__ void atom_exch_16(unsigned long long* p, unsigned long long lo, unsigned long long hi,
+                                             unsigned long long& olo, unsigned long long& ohi) {
+  asm volatile(
+      "{ .reg .b128 d, s; mov.b128 s, {%2, %3}; atom.relaxed.gpu.global.exch.b128 d, [%4], s; "
+      "mov.b128 {%0, %1}, d; }"
+      : "=l"(olo), "=l"(ohi)
+      : "l"(lo), "l"(hi), "l"(p)
+      : "memory");
+}
 __device__ __forceinline__ double ld_relaxed_f64(const double* p) {
   double v;
   asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
@@ -171,20 +194,18 @@ __device__ __forceinline__ double ld_relaxed_f64(const double* p) {
 }
 }  // namespace dev
 
-// Output store.  In a fused exchange (EPI instances with npeer > 0) the element goes to
+// Output store.  In a fused exchange (EPI == 2 instances) the element goes to
 // every rank's copy of the next x over peer memory (NVLink P2P stores through IPC
 // mappings; the rank's own buffer is one of them), so the all-gather overlaps the SpMV.
-template <typename VT, bool EPI>
+template <typename VT, int EPI>
 __device__ __forceinline__ void store_out(const KArgs& a, VT* out, int64_t i, VT v) {
-  if constexpr (EPI) {
-    if (a.npeer > 0) {
+  if constexpr (EPI == 2) {
 #pragma unroll
-      for (int q = 0; q < YASPMV_MAX_RANKS; ++q)
-        if (q < a.npeer) static_cast<VT*>(a.peer_out[q])[i] = v;
-      return;
-    }
+    for (int q = 0; q < YASPMV_MAX_RANKS; ++q)
+      if (q < a.npeer) static_cast<VT*>(a.peer_out[q])[i] = v;
+  } else {
+    out[i] = v;
   }
-  out[i] = v;
 }
 
 template <typename VT, int H, int W, int T, int CM>
@@ -192,6 +213,11 @@ struct KTraits {
   static constexpr int VB = T * W * (int)sizeof(VT);      // value bytes per thread per array
   static constexpr int CB = T * (CM == COL_I32 ? 4 : 2);  // column bytes per thread
   static constexpr int MAXC = (VB * H > 256) ? 256 : 512;
+  // register cap: 96 for the fp32 scalar-row instances (32 values + 32 x in registers) so
+  // that the C5-class kernel keeps 5 CTAs of 128 threads per SM (104 registers would
+  // allow 4: allocation is per warp in units of 8 per thread); otherwise what C <= MAXC
+  // needs (the former __launch_bounds__(MAXC, 1))
+  static constexpr int MAXREG = (sizeof(VT) == 4 && H == 1 && T * W <= 32) ? 96 : (MAXC == 512 ? 128 : 255);
   __host__ __device__ static size_t smem_bytes(int) { return 0; }  // L1 keeps the whole carve-out
 };
 
@@ -205,9 +231,79 @@ struct ScanShared {
   int wn[16];
 };
 
+// Carry-in of tile k's first segment (adjacent synchronization, as a decoupled
+// look-back): the fold of the published tails of tiles k-1, k-2, ... back to the nearest
+// tile holding a row stop (state 2), 32 predecessors per window, fixed association (Q10).
+// Warp-collective; waits only on predecessors nearer than that stop.  Polled with relaxed
+// loads (an acquire would invalidate L1 and with it the cached x); a carry value is read
+// only after its tile's epoch-tagged status word was seen (written before the release).
+template <int H>
+__device__ __forceinline__ void lookback(const KArgs& a, int64_t k, unsigned long long epoch, int lane,
+                                         double (&carry)[H]) {
+#pragma unroll
+  for (int r = 0; r < H; ++r) carry[r] = 0.0;
+  int64_t jw = k - 1;
+  while (true) {
+    const int64_t idx = jw - lane;
+    int state = idx >= 0 ? 0 : 2;  // before tile 0: an inclusive prefix of 0
+    unsigned long long vbits = 0;  // h = 1: the carry-out, read with its status word
+    unsigned p2, lim;
+    while (true) {
+      if (state == 0) {
+        unsigned long long sv;
+        if constexpr (H == 1) dev::ld_relaxed_16(a.status + 2 * idx, sv, vbits);
+        else sv = dev::ld_relaxed(a.status + 2 * idx);
+        if ((sv >> 2) == epoch) state = (int)(sv & 3ull);
+      }
+      p2 = __ballot_sync(0xffffffffu, state == 2);
+      const unsigned p0 = __ballot_sync(0xffffffffu, state == 0);
+      const unsigned nearer = p2 ? ((p2 & (0u - p2)) - 1u) : 0xffffffffu;
+      if ((p0 & nearer) == 0) {
+        lim = p2 ? __ffs(p2) - 1 : 31;  // nearest tile with a row stop
+        break;
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < H; ++r) {
+      double cv = 0.0;
+      if (lane <= (int)lim && idx >= 0) {
+        if constexpr (H == 1) cv = __longlong_as_double((long long)vbits);
+        else cv = dev::ld_relaxed_f64(a.carry + idx * H + r);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) cv += __shfl_xor_sync(0xffffffffu, cv, o);  // fixed tree
+      carry[r] += __shfl_sync(0xffffffffu, cv, 0);
+    }
+    if (p2) break;
+    jw -= 32;
+  }
+}
+
+// y of tile k's carried first segment = (partial + carry-in) scaled; its y^2 partial slot
+template <typename VT, int H, int EPI>
+__device__ __forceinline__ void write_carried(const KArgs& a, VT* out, int64_t k, int64_t row, const double (&dep)[H],
+                                              const double (&carry)[H], double inv, int NW) {
+  double ds = 0.0;
+#pragma unroll
+  for (int r = 0; r < H; ++r)
+    if (row * H + r < a.out_limit) {
+      const VT o = (VT)((dep[r] + carry[r]) * inv);
+      store_out<VT, EPI>(a, out, row * H + r, o);
+      ds += (double)o * (double)o;
+    }
+  if ((EPI == 1 || EPI == 2) && (a.epi & 2)) a.part[k * (NW + 1) + NW] = ds;
+}
+
+// hand-off word tags (bnd[k], per launch epoch): tile k left its carried segment pending /
+// tile k-1 has published its carry-out
+__device__ __forceinline__ unsigned long long bnd_tag(unsigned long long epoch, unsigned who) {
+  return ((epoch & 0x3FFFFFFFull) << 2) | who;  // low 32 bits; h = 1 packs the row above
+}
+constexpr unsigned BND_PENDING = 1, BND_DONE = 2;
+
 // The work of one workgroup-level tile (T*C consecutive blocks): steps 1-3
 // of P:226 plus the cross-tile carry.
-template <typename VT, int H, int W, int T, int CM, bool EPI>
+template <typename VT, int H, int W, int T, int CM, int EPI>
 __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, ScanShared<VT, H>& sh) {
   using TR = KTraits<VT, H, W, T, CM>;
   constexpr int VB = TR::VB, CB = TR::CB;
@@ -227,6 +323,9 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   uint32_t vw[H][VB / 4];
 #pragma unroll
   for (int r = 0; r < H; ++r) dev::load_run<VB>(a.val[r], tile, C, t, pol_s, vw[r]);
+  // the tile's first-result entry: matrix data too, so issued with the stream
+  // instead of after the scan, where its latency would sit on the critical path
+  const int cta_seg0 = __ldg(a.cta_seg0 + tile);
 
   VT* out = static_cast<VT*>(a.out);
   // Programmatic dependent launch: everything above reads only the encoded matrix (never
@@ -237,7 +336,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
     if (a.pdl) cudaGridDependencySynchronize();
     if (t == 0) {
       tk = atomicAdd(a.ticket, 1ull);  // consumed only at the scan barrier (epoch)
-      if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
+      if constexpr (EPI == 1 || EPI == 2) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
     }
   }
   // zero-fill of stacked rows that hold no block (empty_mode MAP, Q1)
@@ -277,7 +376,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
 #pragma unroll
   for (int b = 0; b < T; ++b)
     dev::gather_x<VT, W>(x,
-                         (a.ablate & (ABL_STREAM_ONLY | ABL_GATHER_L2))
+                         (EPI == 3 && (a.ablate & (ABL_STREAM_ONLY | ABL_GATHER_L2)))
                              ? (colb[b] & ((a.ablate & ABL_STREAM_ONLY) ? 15 : 0xFFFFF))
                              : colb[b],
                          a.n, pol_x, xs[b]);
@@ -303,7 +402,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
     }
   }
 
-  if (a.ablate & (ABL_GATHER_ONLY | ABL_STREAM_ONLY)) {  // roofline probes: loads only
+  if (EPI == 3 && (a.ablate & (ABL_GATHER_ONLY | ABL_STREAM_ONLY))) {  // roofline probes: loads only
     VT s = VT(0);
 #pragma unroll
     for (int b = 0; b < T; ++b)
@@ -320,7 +419,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   for (int r = 0; r < H; ++r) v[r] = acc[r];
   const unsigned hs_ballot = __ballot_sync(0xffffffffu, hs);
   // lanes 1..31 all hold a stop: every in-warp segment has size 1 -> skip
-  const bool warp_all_stop = (hs_ballot | 1u) == 0xffffffffu && !(a.ablate & ABL_NO_SKIP);
+  const bool warp_all_stop = (hs_ballot | 1u) == 0xffffffffu && !(EPI == 3 && (a.ablate & ABL_NO_SKIP));
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
     const int f2 = __shfl_up_sync(0xffffffffu, f, d);
@@ -375,21 +474,45 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   VT Vex[H];
 #pragma unroll
   for (int r = 0; r < H; ++r) Vex[r] = fx ? vx[r] : Vw[r] + vx[r];
+  if (EPI == 3 && (a.ablate & ABL_STOP_SCAN)) {  // roofline probe: everything up to the scan
+    if (Vex[0] == VT(-1.25e-30) || Nex == -7) out[t] = Vex[0];
+    return;
+  }
 
   // ---- step 3a: publish this tile's carry-out (adjacent sync) -----------
+  // (thread C-1) the next tile left its carried segment to this one; h = 1: its row and
+  // partial arrive in the exchanged word
+  bool succ_pending = false;
+  unsigned long long succ_lo = 0, succ_hi = 0;
   if (t == C - 1) {
-    double* cv = a.carry + tile * H;
-#pragma unroll
-    for (int r = 0; r < H; ++r) __stcg(cv + r, (double)(hs ? acc[r] : Vex[r] + acc[r]));
     // state 2 = inclusive prefix known (tile holds a stop), 1 = aggregate only
-    dev::st_release(a.status + tile, (epoch << 2) | (Fall ? 2ull : 1ull));
+    const unsigned long long sw = (epoch << 2) | (Fall ? 2ull : 1ull);
+    if constexpr (H == 1) {
+      const double cv0 = (double)(hs ? acc[0] : Vex[0] + acc[0]);
+      dev::st_relaxed_16(a.status + 2 * tile, sw, (unsigned long long)__double_as_longlong(cv0));
+      if constexpr (EPI == 3) __stcg(a.carry + tile, cv0);  // the ablation's carry kernel
+    } else {
+      double* cv = a.carry + tile * H;
+#pragma unroll
+      for (int r = 0; r < H; ++r) __stcg(cv + r, (double)(hs ? acc[r] : Vex[r] + acc[r]));
+      dev::st_release(a.status + 2 * tile, sw);
+    }
+    if (!(EPI == 3 && (a.ablate & ABL_DEFER_CARRY)) && tile + 1 < a.ntiles) {
+      if constexpr (H == 1) {
+        dev::atom_exch_16(a.bnd + 2 * (tile + 1), bnd_tag(epoch, BND_DONE), 0ull, succ_lo, succ_hi);
+        succ_pending = (succ_lo & 0xFFFFFFFFull) == bnd_tag(epoch, BND_PENDING);
+      } else {
+        succ_pending = (dev::atom_exch_acq_rel(a.bnd + 2 * (tile + 1), bnd_tag(epoch, BND_DONE)) & 0xFFFFFFFFull) ==
+                       bnd_tag(epoch, BND_PENDING);
+      }
+    }
   }
 
   // ---- step 2c/3b: combine and write back -----------------------------
   const bool dependent = hs && !Fex && tile > 0;  // the tile's first stop needs the carry
-  const int64_t seg0 = (int64_t)__ldg(a.cta_seg0 + tile) + Nex;  // first-result entry
+  const int64_t seg0 = (int64_t)cta_seg0 + Nex;  // first-result entry
   // optional power-iteration epilogue: y scaled by 1/sqrt(in_norm2), sum y^2 partials
-  const double inv = EPI ? sh.inv : 1.0;
+  const double inv = (EPI == 1 || EPI == 2) ? sh.inv : 1.0;
   const VT invv = (VT)inv;
   VT ssv = VT(0);
   VT dep[H];
@@ -417,9 +540,13 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
 #pragma unroll
             for (int r = 0; r < H; ++r)
               if (H == 1 || row * H + r < a.out_limit) {
-                const VT o = EPI ? run[r] * invv : run[r];
-                store_out<VT, EPI>(a, out, row * H + r, o);
-                if constexpr (EPI) ssv = fma(o, o, ssv);
+                const VT o = (EPI == 1 || EPI == 2) ? run[r] * invv : run[r];
+                if (EPI == 3 && (a.ablate & ABL_NO_YSTORE)) {  // probe: the cost of the y stores
+                  if (o == VT(-1.25e-30)) out[row * H + r] = o;
+                } else {
+                  store_out<VT, EPI>(a, out, row * H + r, o);
+                }
+                if constexpr (EPI == 1 || EPI == 2) ssv = fma(o, o, ssv);
               }
           }
           first = false;
@@ -444,9 +571,9 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
 #pragma unroll
             for (int r = 0; r < H; ++r)
               if (sr * H + r < a.out_limit) {
-                const VT o = EPI ? run[r] * invv : run[r];
+                const VT o = (EPI == 1 || EPI == 2) ? run[r] * invv : run[r];
                 store_out<VT, EPI>(a, out, sr * H + r, o);
-                if constexpr (EPI) ssv = fma(o, o, ssv);
+                if constexpr (EPI == 1 || EPI == 2) ssv = fma(o, o, ssv);
               }
           }
           first = false;
@@ -462,70 +589,88 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   // ---- step 3c: look back for the carry-in (decoupled look-back) --------
   // by the warp holding the tile's first row stop; a window of 32 predecessors per
   // round, polled with relaxed loads (no L1 invalidation: x stays cached in L1)
-  if (EPI && (a.epi & 2)) {  // per-warp partial of sum y^2, fixed tree (deterministic)
+  if ((EPI == 1 || EPI == 2) && (a.epi & 2)) {  // per-warp partial of sum y^2, fixed tree (deterministic)
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
     if (lane == 0) a.part[tile * (NW + 1) + wid] = ss;
     if (t == 0 && !(Fall && tile > 0)) a.part[tile * (NW + 1) + NW] = 0.0;  // no carried segment
   }
-  if (a.ablate & ABL_DEFER_CARRY) {  // ablation: carries by a second kernel
-    if (t == 0 && !(Fall && tile > 0)) a.dep_row[tile] = -1;
+  if (EPI == 3 && (a.ablate & ABL_DEFER_CARRY)) {  // ablation: carries by a second kernel
+    // (dep_row == NULL: the "no carries" probe — the carried segments stay incomplete)
+    if (a.dep_row && t == 0 && !(Fall && tile > 0)) a.dep_row[tile] = -1;
     if (dependent) {
 #pragma unroll
       for (int r = 0; r < H; ++r)
         if (dep_row * H + r < a.out_limit) out[dep_row * H + r] = dep[r];
-      a.dep_row[tile] = dep_row;
+      if (a.dep_row) a.dep_row[tile] = dep_row;
     }
     return;
   }
+  // The warp holding the tile's first row stop needs the carry-in.  Non-blocking hand-off:
+  // if the predecessor has not published yet, leave the partial and its row behind and
+  // exchange the tile's hand-off word; whichever of the two tiles arrives second
+  // completes the segment (the other returns at once), so a tile never holds its SM
+  // slot waiting for a slower predecessor in the common case.  Same arithmetic either
+  // way: (fp64 partial + look-back fold) * inv, rounded once.
   const unsigned dep_ballot = __ballot_sync(0xffffffffu, dependent);
-  if (dep_ballot == 0) return;
-  const int dep_lane = __ffs(dep_ballot) - 1;
-  double carry[H];
+  if (dep_ballot) {
+    const int dep_lane = __ffs(dep_ballot) - 1;
+    unsigned long long sv = 0;
+    if (lane == 0) sv = dev::ld_relaxed(a.status + 2 * (tile - 1));
+    sv = __shfl_sync(0xffffffffu, sv, 0);
+    bool mine = true;
+    const bool can_pack = H > 1 || a.out_limit < (1ll << 32);  // h = 1 packs the row in 32 bits
+    if (((sv >> 2) != epoch || a.force_handoff) && can_pack) {  // predecessor still running: hand off
+      unsigned long long old = 0;
+      if (lane == dep_lane) {
+        if constexpr (H == 1) {
+          unsigned long long ohi;
+          dev::atom_exch_16(a.bnd + 2 * tile, ((unsigned long long)dep_row << 32) | bnd_tag(epoch, BND_PENDING),
+                            (unsigned long long)__double_as_longlong((double)dep[0]), old, ohi);
+        } else {
 #pragma unroll
-  for (int r = 0; r < H; ++r) carry[r] = 0.0;
-  int64_t jw = tile - 1;
-  while (true) {
-    const int64_t idx = jw - lane;
-    int state = 2;  // before tile 0: an inclusive prefix of 0
-    if (idx >= 0) {
-      unsigned long long sv;
-      do { sv = dev::ld_relaxed(a.status + idx); } while ((sv >> 2) != epoch);
-      state = (int)(sv & 3ull);
-    }
-    const unsigned pm = __ballot_sync(0xffffffffu, state == 2);
-    const int lim = pm ? __ffs(pm) - 1 : 31;  // nearest tile with a row stop
-#pragma unroll
-    for (int r = 0; r < H; ++r) {
-      // read only after this lane saw the tile's tagged status word (the value was
-      // written before the release store of that word)
-      double cv = (lane <= lim && idx >= 0) ? dev::ld_relaxed_f64(a.carry + idx * H + r) : 0.0;
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) cv += __shfl_xor_sync(0xffffffffu, cv, o);  // fixed tree
-      carry[r] += __shfl_sync(0xffffffffu, cv, 0);
-    }
-    if (pm) break;
-    jw -= 32;
-  }
-  if (lane == dep_lane) {
-    double ds = 0.0;
-#pragma unroll
-    for (int r = 0; r < H; ++r)
-      if (dep_row * H + r < a.out_limit) {
-        const VT o = (VT)(((double)dep[r] + carry[r]) * inv);
-        store_out<VT, EPI>(a, out, dep_row * H + r, o);
-        ds += (double)o * (double)o;
+          for (int r = 0; r < H; ++r) a.pend_val[tile * H + r] = (double)dep[r];
+          a.pend_row[tile] = dep_row;
+          old = dev::atom_exch_acq_rel(a.bnd + 2 * tile, bnd_tag(epoch, BND_PENDING));
+        }
       }
-    if (EPI && (a.epi & 2)) a.part[tile * (NW + 1) + NW] = ds;
+      old = __shfl_sync(0xffffffffu, old, dep_lane);
+      mine = (old & 0xFFFFFFFFull) == bnd_tag(epoch, BND_DONE);  // it published meanwhile: finish here
+    }
+    if (mine) {
+      double carry[H];
+      lookback<H>(a, tile, epoch, lane, carry);
+      if (lane == dep_lane) {
+        double d[H];
+#pragma unroll
+        for (int r = 0; r < H; ++r) d[r] = (double)dep[r];
+        write_carried<VT, H, EPI>(a, out, tile, dep_row, d, carry, inv, NW);
+      }
+    }
+  }
+  // the next tile handed its carried segment to this one (its predecessor)
+  if (wid == NW - 1 && __shfl_sync(0xffffffffu, succ_pending ? 1 : 0, 31)) {
+    double carry[H];
+    lookback<H>(a, tile + 1, epoch, lane, carry);
+    if (lane == 31) {
+      double d[H];
+      int64_t row;
+      if constexpr (H == 1) {  // carried in the exchanged word
+        d[0] = __longlong_as_double((long long)succ_hi);
+        row = (int64_t)(succ_lo >> 32);
+      } else {  // lane 31's acquire (the exchange) made tile+1's pending data visible
+#pragma unroll
+        for (int r = 0; r < H; ++r) d[r] = a.pend_val[(tile + 1) * H + r];
+        row = (int64_t)a.pend_row[tile + 1];
+      }
+      write_carried<VT, H, EPI>(a, out, tile + 1, row, d, carry, inv, NW);
+    }
   }
 }
 
 // One CTA per workgroup-level tile; logical tile ids from an atomic ticket.
-#ifndef YASPMV_MINB
-#define YASPMV_MINB 1
-#endif
-template <typename VT, int H, int W, int T, int CM, bool EPI>
-__global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) spmv_bccoo_kernel(const KArgs a) {
+template <typename VT, int H, int W, int T, int CM, int EPI>
+__global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_kernel(const KArgs a) {
   __shared__ ScanShared<VT, H> sh;
   if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();  // the next SpMV may start its loads
   if (a.block_ids) {  // tile = workgroup id: workgroups dispatch in order — the default
@@ -538,7 +683,7 @@ __global__ void __launch_bounds__(KTraits<VT, H, W, T, CM>::MAXC, YASPMV_MINB) s
     const unsigned long long q = tk / (unsigned long long)a.period;
     sh.tile = (long long)(tk - q * (unsigned long long)a.period);
     sh.epoch = q + 1ull;  // launches so far: tags this launch's status words (Q9)
-    if constexpr (EPI) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
+    if constexpr (EPI == 1 || EPI == 2) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   }
   __syncthreads();
   tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, sh);
@@ -557,15 +702,22 @@ void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
   attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (a.epi) cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, true>, a);
-  else cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, false>, a);
+  // EPI: 0 plain SpMV, 1 power-iteration epilogue, 2 epilogue + peer stores (fused
+  // exchange), 3 ablation / roofline probes (h = w = 1 only); separate instances so that
+  // neither the peer loop nor the probes cost the production kernel registers
+  if (a.ablate) {
+    if constexpr (H == 1 && W == 1) cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, 3>, a);
+  } else if (a.npeer > 0) cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, 2>, a);
+  else if (a.epi) cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, 1>, a);
+  else cudaLaunchKernelEx(&cfg, spmv_bccoo_kernel<VT, H, W, T, CM, 0>, a);
 }
 
 template <typename VT, int H, int W, int T, int CM>
 int attr_spmv(int C, int* regs, int* max_threads, int* blocks_per_sm) {
   using TR = KTraits<VT, H, W, T, CM>;
-  auto k = spmv_bccoo_kernel<VT, H, W, T, CM, false>;
-  auto k2 = spmv_bccoo_kernel<VT, H, W, T, CM, true>;
+  auto k = spmv_bccoo_kernel<VT, H, W, T, CM, 0>;
+  auto k2 = spmv_bccoo_kernel<VT, H, W, T, CM, 1>;
+  auto k3 = spmv_bccoo_kernel<VT, H, W, T, CM, 2>;
   cudaFuncAttributes fa;
   cudaError_t e = cudaFuncGetAttributes(&fa, k);
   if (e != cudaSuccess) return (int)e;
@@ -584,6 +736,13 @@ int attr_spmv(int C, int* regs, int* max_threads, int* blocks_per_sm) {
     if (e != cudaSuccess) return (int)e;
     e = cudaFuncSetAttribute(k2, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
     if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(k3, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
+    if (e != cudaSuccess) return (int)e;
+    if constexpr (H == 1 && W == 1) {
+      e = cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 3>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                               0);
+      if (e != cudaSuccess) return (int)e;
+    }
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k, C, TR::smem_bytes(C));
     if (e != cudaSuccess) return (int)e;
   }

@@ -96,7 +96,7 @@ def test_integer_exact_random_grid(seed):
             assert np.array_equal(y.astype(np.float64), y_exact), (h, w, T, C, S, cm, em, info)
 
 
-@pytest.mark.parametrize("flags", [0, 8])
+@pytest.mark.parametrize("flags", [0, 8, 32])
 def test_long_row_spanning_many_ctas(flags):
     """One row of 600k entries crosses hundreds of workgroup tiles: carries travel through
     the look-back chain (adjacent synchronization)."""
@@ -154,6 +154,20 @@ def _configs_tolerance(name, flags):
         y, info = _run(csr, x, flags=flags, **p)
         ok, worst = ref.check_tolerance(y, y_ref, bound, dt)
         assert ok, (name, p, worst)
+
+
+@pytest.mark.parametrize("name", ["c1", "c3-ship", "c4"])
+def test_configs_tolerance_forced_handoff(name):
+    """YASPMV_FORCE_HANDOFF: every carried first segment goes through the non-blocking
+    hand-off (tile k leaves its partial, whichever of tiles k-1 / k arrives second finishes
+    it); both finishing sides occur, and y equals the default path bit for bit."""
+    _configs_tolerance(name, 32)
+    csr = synth.config_matrix(name)
+    x = synth.make_x(csr.n, csr.val.dtype, "unit" if name == "c4" else "uniform", 3)
+    for p in CONFIG_PARAMS[name]:
+        y0, _ = _run(csr, x, flags=0, **p)
+        y1, _ = _run(csr, x, flags=32, **p)
+        assert np.array_equal(y0, y1), (name, p)
 
 
 @pytest.mark.parametrize("name", ["c2-f32", "c3-ship", "c4"])

@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--iters", type=int, default=30)
     ap.add_argument("--params", default=None)
     ap.add_argument("--md", default=None)
+    ap.add_argument("--sweep", nargs="*", default=None, help="JSON param overrides, one re-encode each")
     args = ap.parse_args()
     import torch
 
@@ -40,12 +41,24 @@ def main():
     params = dict(DEFAULT_PARAMS.get(args.config, {}))
     if args.params:
         params.update(json.loads(args.params))
+    sweep = [json.loads(p) for p in args.sweep] if args.sweep else [{}]
     if csr.nnz > 50_000_000:
-        params.setdefault("flags", 2 | 4)
+        params.setdefault("flags", 4 if len(sweep) > 1 else 2 | 4)
     A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=0, **params)
-    info = A.info()
     nnz = csr.nnz
     del csr
+    for sw in sweep:
+        if sw:
+            A.reencode(**sw)
+        _probe(A, nnz, args)
+    A.free()
+
+
+def _probe(A, nnz, args):
+    import torch
+    from paper_conf_ppopp_yanlzz14_b200._lib import check, lib
+    from bench import measured_peaks
+    info = A.info()
     x = torch.full((info["n"],), 1.0 / np.sqrt(info["n"]), dtype=torch.float32 if A.dtype == np.float32
                    else torch.float64, device="cuda")
     y = torch.zeros(info["m"], dtype=x.dtype, device="cuda")
@@ -59,7 +72,9 @@ def main():
             check(lib.yaspmv_ablation_spmv(A._h, variant, x.data_ptr(), y.data_ptr(), st))
 
     out = []
-    probes = [("full", 0), ("stream+gather", 4), ("stream+L2-gather", 6), ("stream", 5), ("full (again)", 0)]
+    probes = [("full", 0), ("no carries (7)", 7), ("7 - y stores (9)", 9),
+              ("up to the scan (8)", 8), ("stream+gather", 4),
+              ("stream+L2-gather", 6), ("stream", 5), ("full (again)", 0)]
     for name, v in probes:
         if v == 6 and info["n"] < (1 << 20) * info["params"]["block_w"]:
             continue
@@ -80,13 +95,13 @@ def main():
         out.append(line)
         print(json.dumps(line), flush=True)
     if args.md:
-        with open(args.md, "w") as f:
+        with open(args.md, "a") as f:
             f.write(f"# K1 roofline probes — {args.config} ({nnz:,} nnz), params {info['params']}\n\n")
             f.write("| probe | ms | GFLOPS-equiv | algorithmic GB/s | frac of measured HBM |\n|---|---|---|---|---|\n")
             for r in out:
                 f.write(f"| {r['probe']} | {r['ms']:.3f} | {r['gflops_equiv']:.0f} | {r['alg_gbs']:.0f} | "
                         f"{r['alg_frac']:.3f} |\n")
-    A.free()
+            f.write("\n")
 
 
 if __name__ == "__main__":
