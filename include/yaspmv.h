@@ -74,6 +74,13 @@ typedef struct {
   int32_t col_mode;    /* YASPMV_COL_*; U16 requires ceil(n/w) < 65535           */
   int32_t empty_mode;  /* YASPMV_EMPTY_*                                                  */
   int32_t flags;       /* YASPMV_KEEP_HOST | YASPMV_DROP_CSR | YASPMV_GPU_ENCODE         */
+  int32_t result_cache; /* segmented-sum strategy (Table 1; §3.2.2-3.2.3):
+                           0 = strategy 1 (intermediate sums in registers);
+                           k in {1,2,4} = strategy 2 with a per-workgroup result cache of
+                           k*C entries in shared memory, written back coalesced (P:274-278,
+                           P:293).  Results agree within rounding (the first stop's sum is
+                           associated differently).  yaspmv_reencode: 0 = keep current,
+                           -1 = strategy 1.  A launch-time choice: no re-encode needed. */
 } yaspmv_params;
 
 typedef struct {
@@ -167,7 +174,9 @@ yaspmv_status yaspmv_host_sync(yaspmv_matrix A);
 /* ---------------------------------------------------------------- tuning (§4)
  * yaspmv_tune: auto-tuner of PAPER.md §4: for the 4 block shapes with the
  * smallest footprint it times the SpMV over thread tile T, CTA size C, slice count
- * S and column mode on the device (scratch x/y owned by the tuner), then re-encodes A with
+ * S and column mode with strategy 1, then strategy 2 with result cache sizes 1 and 2 (the
+ * paper's pinned values) for the two fastest (T, C) of each (h, w, S, col mode), on
+ * the device (scratch x/y owned by the tuner), then re-encodes A with
  * the fastest parameters (ties within 1%: smaller footprint, then lexicographic).
  * Re-encoding needs the normalised CSR the handle keeps unless built with
  * YASPMV_DROP_CSR (then EINVAL).  On failure A keeps its previous parameters.
@@ -178,7 +187,8 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen);
  * against). */
 yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode);
 
-/* yaspmv_reencode: re-encode A with new parameters (0 fields = keep current). */
+/* yaspmv_reencode: re-encode A with new parameters (0 fields = keep current; see
+ * result_cache for its -1).  A change of result_cache alone only re-selects the kernel. */
 yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params);
 
 /* ---------------------------------------------------------------- introspection

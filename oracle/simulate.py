@@ -12,7 +12,9 @@ Follows PAPER.md §3.2 in the paper's order and notation:
   * combine: the first stop of thread t adds last_partial_sums[t-1] (scanned), and the
     previous workgroup's Grp_sum when the segment spans workgroups (§3.2.3, P:287-292);
   * adjacent synchronization: Grp_sum[X] = last partial sum of X if X holds a row stop,
-    else Grp_sum[X-1] + last partial sum of X (§3.2.4).
+    else Grp_sum[X-1] + last partial sum of X (§3.2.4, P:297-298);
+  * simulate_s2: strategy 2, the per-workgroup result cache addressed by first-result
+    entries (§3.2.2, §3.2.3, Figs. 10/12).
 Generic over the element type (ints, Fractions, floats): no rounding of its own.
 """
 from __future__ import annotations
@@ -80,4 +82,80 @@ def simulate(values, bits, T: int, C: int):
                 results.append(v)
         trace.append({"last_partial_sums": lps, "start_flags": start, "scanned": scanned,
                       "grp_sum": grp, "skip_scan": all(start[1:])})
+    return results, trace
+
+
+def simulate_s2(values, bits, T: int, C: int, RC: int):
+    """Strategy 2 (§3.2.2, §3.2.3, Figs. 10 and 12), same inputs as
+    simulate() plus RC = result cache entries per workgroup (Table 1: a multiple of the
+    workgroup size).  Per workgroup, in the paper's order:
+      * first-result entries (P:189): fre[t] = row stops in the tile before thread t;
+      * each thread runs its sequential segmented sum over its tile; at each row stop the
+        current sum goes to result-cache entry fre[t] + j (j-th stop of the thread), or to
+        the global result array when that entry is >= RC ("larger than the results cache
+        size", P:278); its last partial sum goes to last_partial_sums (P:278);
+      * the parallel segmented scan of last_partial_sums (P:282);
+      * each thread except thread 0 that has a stop adds last_partial_sums[t-1] (scanned)
+        to its first entry; thread 0 adds the previous workgroup's Grp_sum to entry 0 (and
+        so does any thread whose first stop is the workgroup's first, i.e. no earlier
+        thread of the workgroup had a stop) — the "segments spanning workgroups" case;
+      * the cache (and the overflow entries) are the workgroup's segment sums, in order.
+    Returns (segment_sums, trace); trace holds per workgroup the cache right after the
+    threads' walks ("cache_walk"), after the fix-up ("cache"), and fre."""
+    n = len(values)
+    assert n % (T * C) == 0 and len(bits) == n and RC >= 1
+    zero = values[0] * 0 if n else 0
+    results = []
+    trace = []
+    grp_sum = []
+    for X in range(n // (T * C)):
+        base = X * T * C
+        nst = [sum(1 for i in range(T) if bits[base + t * T + i] == 0) for t in range(C)]
+        fre = [sum(nst[:t]) for t in range(C)]
+        total = sum(nst)
+        cache = [None] * min(RC, total)
+        overflow = {}                  # entry -> value, entries >= RC (global result array)
+        lps, start = [], []
+        for t in range(C):
+            s = zero
+            j = 0
+            for i in range(T):
+                b = base + t * T + i
+                s = s + values[b]
+                if bits[b] == 0:
+                    e = fre[t] + j
+                    if e < RC:
+                        cache[e] = s
+                    else:
+                        overflow[e] = s
+                    j += 1
+                    s = zero
+            lps.append(s)
+            start.append(1 if j else 0)
+        cache_walk = list(cache)
+        scanned = []
+        for t in range(C):
+            scanned.append(lps[t] if (t == 0 or start[t]) else scanned[t - 1] + lps[t])
+        if any(start):
+            grp = scanned[C - 1]
+        else:
+            grp = (grp_sum[X - 1] if X > 0 else zero) + scanned[C - 1]
+        prev_grp = grp_sum[X - 1] if X > 0 else zero
+        grp_sum.append(grp)
+        for t in range(C):
+            if not start[t]:
+                continue
+            e = fre[t]
+            v = cache[e] if e < RC else overflow[e]
+            if t > 0:
+                v = scanned[t - 1] + v
+            if not any(start[:t]):
+                v = prev_grp + v
+            if e < RC:
+                cache[e] = v
+            else:
+                overflow[e] = v
+        results.extend(cache[e] if e < RC else overflow[e] for e in range(total))
+        trace.append({"fre": fre, "cache_walk": cache_walk, "cache": list(cache), "last_partial_sums": lps,
+                      "scanned": scanned, "grp_sum": grp})
     return results, trace

@@ -55,6 +55,7 @@ Params from_abi(const yaspmv_params* p) {
     q.col_mode = p->col_mode;
     q.empty_mode = p->empty_mode;
     q.flags = p->flags;
+    q.rc = p->result_cache;
   }
   return q;
 }
@@ -69,6 +70,7 @@ yaspmv_params to_abi(const Params& q) {
   p.col_mode = q.col_mode;
   p.empty_mode = q.empty_mode;
   p.flags = q.flags;
+  p.result_cache = q.rc;
   return p;
 }
 
@@ -163,11 +165,11 @@ yaspmv_status to_device(yaspmv_matrix A) {
 yaspmv_status select_kernel(yaspmv_matrix A) {
   const Params& p = A->can.p;
   if (A->device < 0) return YASPMV_OK;  // host-only handles never launch
-  A->kern = find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode);
+  A->kern = find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode, p.rc > 0 ? 2 : 1);
   if (!A->kern)
     return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for dtype/h/w/T (values per thread exceed 512 bytes)");
   int regs = 0, maxt = 0, bps = 0;
-  int e = A->kern->attr(p.C, &regs, &maxt, &bps);
+  int e = A->kern->attr(p.C, p.rc, &regs, &maxt, &bps);
   if (e != 0) return fail(YASPMV_ECUDA, std::string("kernel attributes: ") + cudaGetErrorString((cudaError_t)e));
   if (p.C > maxt) return fail(YASPMV_EUNSUPPORTED, "cta_size exceeds the kernel's launch bound");
   if (bps <= 0) return fail(YASPMV_EUNSUPPORTED, "kernel does not fit on an SM with this cta_size");
@@ -220,7 +222,7 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
   Params p;
   yaspmv_status st = resolve_params(want, A->csr.m, A->csr.n, p);
   if (st != YASPMV_OK) return st;
-  if (A->device >= 0 && !find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode))
+  if (A->device >= 0 && !find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode, p.rc > 0 ? 2 : 1))
     return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for this (dtype, h, w, T): values per thread > 512 B");
   if ((p.flags & YASPMV_GPU_ENCODE) && A->device >= 0) {
     CUDA_TRY(cudaSetDevice(A->device));
@@ -371,6 +373,8 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   a.dep_row = nullptr;
   a.npeer = 0;
   for (int q = 0; q < YASPMV_MAX_RANKS; ++q) a.peer_out[q] = nullptr;
+  a.rcache = p.rc * p.C;
+  if (ablate && p.rc > 0) return fail(YASPMV_EUNSUPPORTED, "ablation / probe variants are strategy-1 kernels");
   if (peers && p.S == 1) {  // S > 1: the kernel writes tmp, the combine writes the peers
     a.npeer = peers->n;
     for (int q = 0; q < peers->n; ++q) a.peer_out[q] = peers->p[q];
@@ -406,6 +410,21 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
 }
 
 }  // namespace
+
+// switch the segmented-sum strategy of an encoded handle (kernel re-selection only)
+yaspmv_status set_strategy(yaspmv_matrix A, int rc) {
+  const int old = A->can.p.rc;
+  const KernelEntry* oldk = A->kern;
+  const int64_t oldgrid = A->grid;
+  A->can.p.rc = rc;
+  yaspmv_status st = select_kernel(A);
+  if (st != YASPMV_OK) {
+    A->can.p.rc = old;
+    A->kern = oldk;
+    A->grid = oldgrid;
+  }
+  return st;
+}
 
 yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags) {
   return install_canonical_impl(A, std::move(c), flags);
@@ -473,6 +492,14 @@ yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
   if (!want.T) want.T = cur.T;
   if (!want.C) want.C = cur.C;
   if (!params) want.flags = cur.flags;
+  want.rc = want.rc == 0 ? cur.rc : (want.rc < 0 ? 0 : want.rc);
+  {  // only the strategy changes: a launch-time choice, no re-encode (Table 1 axes T..S unchanged)
+    Params rp;
+    if (A->device >= 0 && resolve_params(want, A->csr.m, A->csr.n, rp) == YASPMV_OK && rp.h == cur.h &&
+        rp.w == cur.w && rp.S == cur.S && rp.T == cur.T && rp.C == cur.C && rp.col_mode == cur.col_mode &&
+        (rp.empty_mode == 0 || rp.empty_mode == cur.empty_mode) && rp.flags == cur.flags)
+      return set_strategy(A, rp.rc);
+  }
   return encode_into(A, want);
 }
 

@@ -247,7 +247,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             const int64_t tiles = (nnzb_est + (int64_t)T * C - 1) / ((int64_t)T * C);
             if (tiles < 2 * sms && (T * C) > 1024) continue;
             if (gpu) {
-              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode, YASPMV_GPU_ENCODE};
+              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode, YASPMV_GPU_ENCODE, -1};
               if (yaspmv_reencode(A, &ap) != YASPMV_OK) continue;
             } else {
               Canonical cand;
@@ -271,6 +271,28 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             yaspmv_info info;
             yaspmv_get_info(A, &info);
             results.push_back({ts[ts.size() / 2], info.format_bytes, A->can.p});
+            // strategy 2 with the paper's pinned result cache sizes 1 and 2: a
+            // launch-time switch on the same encoding
+            for (int rc : {1, 2}) {
+              if (!find_kernel(A->dtype, sh.h, sh.w, T, cm, 2) || set_strategy(A, rc) != YASPMV_OK) continue;
+              bool ok2 = true;
+              for (int it = 0; it < 3 && ok2; ++it) ok2 = yaspmv_spmv(A, x, y, stream) == YASPMV_OK;
+              if (ok2) {
+                std::vector<float> t2;
+                for (int it = 0; it < 7; ++it) {
+                  cudaEventRecord(e0, st);
+                  yaspmv_spmv(A, x, y, stream);
+                  cudaEventRecord(e1, st);
+                  cudaEventSynchronize(e1);
+                  float ms = 0;
+                  cudaEventElapsedTime(&ms, e0, e1);
+                  t2.push_back(ms);
+                }
+                std::sort(t2.begin(), t2.end());
+                results.push_back({t2[t2.size() / 2], info.format_bytes, A->can.p});
+              }
+              set_strategy(A, 0);
+            }
           }
         }
       }
@@ -281,7 +303,8 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   cudaFree(x);
   cudaFree(y);
   if (results.empty()) {
-    yaspmv_params back{saved.h, saved.w, saved.S, saved.T, saved.C, saved.col_mode, saved.empty_mode, keep_flags};
+    yaspmv_params back{saved.h, saved.w, saved.S, saved.T, saved.C, saved.col_mode, saved.empty_mode, keep_flags,
+                       saved.rc > 0 ? saved.rc : -1};
     yaspmv_reencode(A, &back);
     return fail(YASPMV_EUNSUPPORTED, "no tunable candidate could be launched");
   }
@@ -292,18 +315,18 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   for (const Cand& c : results) {
     if (c.ms > best_ms * 1.01f) continue;
     if (!best) { best = &c; continue; }
-    auto key = [](const Cand& q) { return std::make_tuple(q.bytes, q.p.h, q.p.w, q.p.T, q.p.C, q.p.S); };
+    auto key = [](const Cand& q) { return std::make_tuple(q.bytes, q.p.h, q.p.w, q.p.T, q.p.C, q.p.S, q.p.rc); };
     if (key(c) < key(*best)) best = &c;
   }
   yaspmv_params bp{best->p.h, best->p.w, best->p.S, best->p.T, best->p.C, best->p.col_mode, best->p.empty_mode,
-                   keep_flags};
+                   keep_flags, best->p.rc > 0 ? best->p.rc : -1};
   yaspmv_status rs = yaspmv_reencode(A, &bp);
   if (rs != YASPMV_OK) return rs;
   A->tune_s = now_s() - t0;
   A->tune_candidates = (int)results.size();
   if (chosen) {
     const Params& q = A->can.p;
-    *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags};
+    *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags, q.rc};
   }
   return YASPMV_OK;
 }

@@ -29,6 +29,7 @@ enum Ablate {
 
 struct Params {
   int h = 1, w = 1, S = 1, T = 16, C = 256, col_mode = 0, empty_mode = 0, flags = 0;
+  int rc = 0;  // result cache size in units of C: 0 = strategy 1, k > 0 = strategy 2 (Table 1)
 };
 
 inline int col_bytes(int mode) { return mode == COL_I32 ? 4 : 2; }
@@ -152,6 +153,7 @@ struct KArgs {
   // pre-offset to this rank's chunk) instead of out[i]
   int npeer;
   void* peer_out[YASPMV_MAX_RANKS];
+  int rcache;              // strategy 2: result cache entries (rc * C); 0 for strategy 1
 };
 
 // destinations of a fused exchange (combine kernel of BCCOO+, S > 1)
@@ -161,15 +163,16 @@ struct PeerOut {
 };
 
 typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
-typedef int (*AttrFn)(int C, int* regs, int* max_threads, int* blocks_per_sm);
+typedef int (*AttrFn)(int C, int rc, int* regs, int* max_threads, int* blocks_per_sm);
 
 struct KernelEntry {
   int dtype, h, w, T, cm;
+  int strat;  // segmented-sum strategy (P:267 / P:274): 1 registers, 2 result cache
   LaunchFn launch;
   AttrFn attr;
 };
 
-const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm);
+const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm, int strat = 1);
 const std::vector<KernelEntry>& all_kernels();
 
 void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream,

@@ -193,6 +193,9 @@ yaspmv_status resolve_params(const Params& in, int64_t m, int64_t n, Params& out
   if (out.col_mode == COL_U16 && NB >= 65535)
     return fail(YASPMV_EINVAL, "u16 column storage needs ceil(n/w) < 65535 (P:302)");
   if (out.empty_mode < 0 || out.empty_mode > 2) return fail(YASPMV_EINVAL, "bad empty_mode");
+  if (out.rc < 0) out.rc = 0;  // -1 = strategy 1 explicitly (yaspmv_reencode)
+  if (out.rc != 0 && out.rc != 1 && out.rc != 2 && out.rc != 4)
+    return fail(YASPMV_EINVAL, "result_cache must be 0 (strategy 1) or 1, 2, 4 (x C entries, strategy 2)");
   (void)m;
   return YASPMV_OK;
 }

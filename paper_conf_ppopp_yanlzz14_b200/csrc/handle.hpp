@@ -95,3 +95,5 @@ yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags);
 // of a local y (the fused exchange of comm.cu); out_norm2 receives sum y^2 (nullable)
 yaspmv_status run_spmv_peers(yaspmv_matrix A, const void* x, const double* in_norm2, double* out_norm2,
                              const yaspmv::PeerOut& peers, void* stream);
+// capi.cpp: switch the segmented-sum strategy (result_cache) of an encoded handle
+yaspmv_status set_strategy(yaspmv_matrix A, int rc);

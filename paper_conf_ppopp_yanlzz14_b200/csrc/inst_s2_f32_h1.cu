@@ -1,0 +1,8 @@
+// Precompiled strategy-2 SpMV kernel instances (result cache, Table 1):
+// dtype float, block height 1, block widths {1,2,4,8} x thread tiles {4,8,16,32} x column
+// modes, restricted to T*h*w*sizeof(value) <= 512 bytes of values per thread.
+#include "spmv_kernel.cuh"
+
+namespace yaspmv {
+void register_s2_f32_h1(std::vector<KernelEntry>& R) { reg_h_s2<float, 1>(R); }
+}  // namespace yaspmv

@@ -169,6 +169,14 @@ void register_f64_h1(std::vector<KernelEntry>&);
 void register_f64_h2(std::vector<KernelEntry>&);
 void register_f64_h3(std::vector<KernelEntry>&);
 void register_f64_h4(std::vector<KernelEntry>&);
+void register_s2_f32_h1(std::vector<KernelEntry>&);
+void register_s2_f32_h2(std::vector<KernelEntry>&);
+void register_s2_f32_h3(std::vector<KernelEntry>&);
+void register_s2_f32_h4(std::vector<KernelEntry>&);
+void register_s2_f64_h1(std::vector<KernelEntry>&);
+void register_s2_f64_h2(std::vector<KernelEntry>&);
+void register_s2_f64_h3(std::vector<KernelEntry>&);
+void register_s2_f64_h4(std::vector<KernelEntry>&);
 
 const std::vector<KernelEntry>& all_kernels() {
   static std::vector<KernelEntry> R;
@@ -182,13 +190,21 @@ const std::vector<KernelEntry>& all_kernels() {
     register_f64_h2(R);
     register_f64_h3(R);
     register_f64_h4(R);
+    register_s2_f32_h1(R);
+    register_s2_f32_h2(R);
+    register_s2_f32_h3(R);
+    register_s2_f32_h4(R);
+    register_s2_f64_h1(R);
+    register_s2_f64_h2(R);
+    register_s2_f64_h3(R);
+    register_s2_f64_h4(R);
   });
   return R;
 }
 
-const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm) {
+const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm, int strat) {
   for (const KernelEntry& e : all_kernels())
-    if (e.dtype == dtype && e.h == h && e.w == w && e.T == T && e.cm == cm) return &e;
+    if (e.dtype == dtype && e.h == h && e.w == w && e.T == T && e.cm == cm && e.strat == strat) return &e;
   return nullptr;
 }
 

@@ -301,37 +301,136 @@ __device__ __forceinline__ unsigned long long bnd_tag(unsigned long long epoch, 
 }
 constexpr unsigned BND_PENDING = 1, BND_DONE = 2;
 
-// The work of one workgroup-level tile (T*C consecutive blocks, P:259-262): steps 1-3
-// of P:226 plus the cross-tile carry (P:295-298).
+// Step 3a of a tile (thread C-1): publish the tile's carry-out — its status word with the
+// inclusive value when the tile holds a row stop (the paper's "directly updates"),
+// else its aggregate — and take over the successor's carried segment if the successor
+// already left it behind (non-blocking hand-off, see resolve_carries).
+template <typename VT, int H, int EPI>
+__device__ __forceinline__ void publish_carry(const KArgs& a, const int64_t tile, const unsigned long long epoch,
+                                              const int Fall, const int hs, const VT (&acc)[H], const VT (&Vex)[H],
+                                              bool& succ_pending, unsigned long long& succ_lo,
+                                              unsigned long long& succ_hi) {
+  // state 2 = inclusive prefix known (tile holds a stop), 1 = aggregate only
+  const unsigned long long sw = (epoch << 2) | (Fall ? 2ull : 1ull);
+  if constexpr (H == 1) {
+    const double cv0 = (double)(hs ? acc[0] : Vex[0] + acc[0]);
+    dev::st_relaxed_16(a.status + 2 * tile, sw, (unsigned long long)__double_as_longlong(cv0));
+    if constexpr (EPI == 3) __stcg(a.carry + tile, cv0);  // the ablation's carry kernel
+  } else {
+    double* cv = a.carry + tile * H;
+#pragma unroll
+    for (int r = 0; r < H; ++r) __stcg(cv + r, (double)(hs ? acc[r] : Vex[r] + acc[r]));
+    dev::st_release(a.status + 2 * tile, sw);
+  }
+  if (!(EPI == 3 && (a.ablate & ABL_DEFER_CARRY)) && tile + 1 < a.ntiles) {
+    if constexpr (H == 1) {
+      dev::atom_exch_16(a.bnd + 2 * (tile + 1), bnd_tag(epoch, BND_DONE), 0ull, succ_lo, succ_hi);
+      succ_pending = (succ_lo & 0xFFFFFFFFull) == bnd_tag(epoch, BND_PENDING);
+    } else {
+      succ_pending = (dev::atom_exch_acq_rel(a.bnd + 2 * (tile + 1), bnd_tag(epoch, BND_DONE)) & 0xFFFFFFFFull) ==
+                     bnd_tag(epoch, BND_PENDING);
+    }
+  }
+}
+
+// Step 3c of a tile: the carry-in of its first row stop (decoupled look-back) and the
+// successor's carried segment if it was handed to this tile.
+template <typename VT, int H, int EPI>
+__device__ __forceinline__ void resolve_carries(const KArgs& a, VT* out, const int64_t tile,
+                                                const unsigned long long epoch, const int lane, const int wid,
+                                                const int NW, const bool dependent, const VT (&dep)[H],
+                                                const int64_t dep_row, const double inv, const bool succ_pending,
+                                                const unsigned long long succ_lo, const unsigned long long succ_hi) {
+  // The warp holding the tile's first row stop needs the carry-in.  Non-blocking hand-off:
+  // if the predecessor has not published yet, leave the partial and its row behind and
+  // exchange the tile's hand-off word; whichever of the two tiles arrives second
+  // completes the segment (the other returns at once), so a tile never holds its SM
+  // slot waiting for a slower predecessor in the common case.  Same arithmetic either
+  // way: (fp64 partial + look-back fold) * inv, rounded once.
+  const unsigned dep_ballot = __ballot_sync(0xffffffffu, dependent);
+  if (dep_ballot) {
+    const int dep_lane = __ffs(dep_ballot) - 1;
+    unsigned long long sv = 0;
+    if (lane == 0) sv = dev::ld_relaxed(a.status + 2 * (tile - 1));
+    sv = __shfl_sync(0xffffffffu, sv, 0);
+    bool mine = true;
+    const bool can_pack = H > 1 || a.out_limit < (1ll << 32);  // h = 1 packs the row in 32 bits
+    if (((sv >> 2) != epoch || a.force_handoff) && can_pack) {  // predecessor still running: hand off
+      unsigned long long old = 0;
+      if (lane == dep_lane) {
+        if constexpr (H == 1) {
+          unsigned long long ohi;
+          dev::atom_exch_16(a.bnd + 2 * tile, ((unsigned long long)dep_row << 32) | bnd_tag(epoch, BND_PENDING),
+                            (unsigned long long)__double_as_longlong((double)dep[0]), old, ohi);
+        } else {
+#pragma unroll
+          for (int r = 0; r < H; ++r) a.pend_val[tile * H + r] = (double)dep[r];
+          a.pend_row[tile] = dep_row;
+          old = dev::atom_exch_acq_rel(a.bnd + 2 * tile, bnd_tag(epoch, BND_PENDING));
+        }
+      }
+      old = __shfl_sync(0xffffffffu, old, dep_lane);
+      mine = (old & 0xFFFFFFFFull) == bnd_tag(epoch, BND_DONE);  // it published meanwhile: finish here
+    }
+    if (mine) {
+      double carry[H];
+      lookback<H>(a, tile, epoch, lane, carry);
+      if (lane == dep_lane) {
+        double d[H];
+#pragma unroll
+        for (int r = 0; r < H; ++r) d[r] = (double)dep[r];
+        write_carried<VT, H, EPI>(a, out, tile, dep_row, d, carry, inv, NW);
+      }
+    }
+  }
+  // the next tile handed its carried segment to this one (its predecessor)
+  if (wid == NW - 1 && __shfl_sync(0xffffffffu, succ_pending ? 1 : 0, 31)) {
+    double carry[H];
+    lookback<H>(a, tile + 1, epoch, lane, carry);
+    if (lane == 31) {
+      double d[H];
+      int64_t row;
+      if constexpr (H == 1) {  // carried in the exchanged word
+        d[0] = __longlong_as_double((long long)succ_hi);
+        row = (int64_t)(succ_lo >> 32);
+      } else {  // lane 31's acquire (the exchange) made tile+1's pending data visible
+#pragma unroll
+        for (int r = 0; r < H; ++r) d[r] = a.pend_val[(tile + 1) * H + r];
+        row = (int64_t)a.pend_row[tile + 1];
+      }
+      write_carried<VT, H, EPI>(a, out, tile + 1, row, d, carry, inv, NW);
+    }
+  }
+}
+
+// Step 1 of a tile: stream the thread tile — bit flags,
+// block columns, values (128-bit loads of the offline-transposed layout, L2 evict-first)
+// and the tile's first-result entry — then, after the programmatic-dependent-launch wait,
+// take the epoch ticket, zero-fill empty stacked rows (Q1) and issue all T gathers of x.
 template <typename VT, int H, int W, int T, int CM, int EPI>
-__device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, ScanShared<VT, H>& sh) {
+__device__ __forceinline__ void stream_tile(const KArgs& a, const int64_t tile, ScanShared<VT, H>& sh, const int t,
+                                            const int C, uint32_t& fl,
+                                            uint32_t (&vw)[H][KTraits<VT, H, W, T, CM>::VB / 4], VT (&xs)[T][W],
+                                            int& cta_seg0, unsigned long long& tk) {
   using TR = KTraits<VT, H, W, T, CM>;
   constexpr int VB = TR::VB, CB = TR::CB;
-  constexpr uint32_t TMASK = (T == 32) ? 0xffffffffu : ((1u << T) - 1u);
-  auto& s_wv = sh.wv;
-  auto& s_wf = sh.wf;
-  auto& s_wn = sh.wn;
-  const int t = threadIdx.x, C = blockDim.x, lane = t & 31, wid = t >> 5, NW = C >> 5;
   const uint64_t pol_s = dev::policy_evict_first();
   const uint64_t pol_x = dev::policy_evict_last();
-
   // ---- step 1: stream the thread tile (128-bit loads, offline-transposed layout) ----
   const int64_t blk0 = tile * (int64_t)C * T + (int64_t)t * T;
-  const uint32_t fl = dev::load_flags<T>(a.flags, blk0);
+  fl = dev::load_flags<T>(a.flags, blk0);
   uint32_t cw[CB / 4];
   dev::load_run<CB>(a.col, tile, C, t, pol_s, cw);
-  uint32_t vw[H][VB / 4];
 #pragma unroll
   for (int r = 0; r < H; ++r) dev::load_run<VB>(a.val[r], tile, C, t, pol_s, vw[r]);
   // the tile's first-result entry: matrix data too, so issued with the stream
   // instead of after the scan, where its latency would sit on the critical path
-  const int cta_seg0 = __ldg(a.cta_seg0 + tile);
+  cta_seg0 = __ldg(a.cta_seg0 + tile);
 
   VT* out = static_cast<VT*>(a.out);
   // Programmatic dependent launch: everything above reads only the encoded matrix (never
   // written by other kernels) and overlaps the previous kernel's tail; x, y, the status
   // words and the ticket may depend on earlier kernels in the stream.
-  unsigned long long tk = 0;
   if (a.block_ids) {
     if (a.pdl) cudaGridDependencySynchronize();
     if (t == 0) {
@@ -350,11 +449,6 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
         if (sr * H + r < a.out_limit) store_out<VT, EPI>(a, out, sr * H + r, VT(0));
     }
   }
-  // row stops: '0' bits (P:114); one popc gives their count (P:262)
-  const uint32_t stops = ~fl & TMASK;
-  const int nst = __popc(stops);
-  const int hs = nst > 0;
-
   // block columns, then all T gathers of x in flight
   int colb[T];
 #pragma unroll
@@ -372,7 +466,6 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
     }
   }
   const VT* x = static_cast<const VT*>(a.x);
-  VT xs[T][W];
 #pragma unroll
   for (int b = 0; b < T; ++b)
     dev::gather_x<VT, W>(x,
@@ -380,6 +473,31 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
                              ? (colb[b] & ((a.ablate & ABL_STREAM_ONLY) ? 15 : 0xFFFFF))
                              : colb[b],
                          a.n, pol_x, xs[b]);
+}
+
+// The work of one workgroup-level tile (T*C consecutive blocks, P:259-262): steps 1-3
+// of P:226 plus the cross-tile carry (P:295-298).
+template <typename VT, int H, int W, int T, int CM, int EPI>
+__device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, ScanShared<VT, H>& sh) {
+  using TR = KTraits<VT, H, W, T, CM>;
+  constexpr int VB = TR::VB;
+  constexpr uint32_t TMASK = (T == 32) ? 0xffffffffu : ((1u << T) - 1u);
+  auto& s_wv = sh.wv;
+  auto& s_wf = sh.wf;
+  auto& s_wn = sh.wn;
+  const int t = threadIdx.x, C = blockDim.x, lane = t & 31, wid = t >> 5, NW = C >> 5;
+  // ---- step 1: stream the thread tile, gather x ------------------------------------
+  uint32_t fl;
+  uint32_t vw[H][VB / 4];
+  VT xs[T][W];
+  int cta_seg0;
+  unsigned long long tk = 0;
+  stream_tile<VT, H, W, T, CM, EPI>(a, tile, sh, t, C, fl, vw, xs, cta_seg0, tk);
+  VT* out = static_cast<VT*>(a.out);
+  // row stops: '0' bits (P:114); one popc gives their count (P:262)
+  const uint32_t stops = ~fl & TMASK;
+  const int nst = __popc(stops);
+  const int hs = nst > 0;
 
   // ---- step 2a: multiply + per-thread sequential segmented sum ------
   // Strategy 1: the per-block products stay in registers ("intermediate_sums",
@@ -480,33 +598,9 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   }
 
   // ---- step 3a: publish this tile's carry-out (adjacent sync) -----------
-  // (thread C-1) the next tile left its carried segment to this one; h = 1: its row and
-  // partial arrive in the exchanged word
   bool succ_pending = false;
   unsigned long long succ_lo = 0, succ_hi = 0;
-  if (t == C - 1) {
-    // state 2 = inclusive prefix known (tile holds a stop), 1 = aggregate only
-    const unsigned long long sw = (epoch << 2) | (Fall ? 2ull : 1ull);
-    if constexpr (H == 1) {
-      const double cv0 = (double)(hs ? acc[0] : Vex[0] + acc[0]);
-      dev::st_relaxed_16(a.status + 2 * tile, sw, (unsigned long long)__double_as_longlong(cv0));
-      if constexpr (EPI == 3) __stcg(a.carry + tile, cv0);  // the ablation's carry kernel
-    } else {
-      double* cv = a.carry + tile * H;
-#pragma unroll
-      for (int r = 0; r < H; ++r) __stcg(cv + r, (double)(hs ? acc[r] : Vex[r] + acc[r]));
-      dev::st_release(a.status + 2 * tile, sw);
-    }
-    if (!(EPI == 3 && (a.ablate & ABL_DEFER_CARRY)) && tile + 1 < a.ntiles) {
-      if constexpr (H == 1) {
-        dev::atom_exch_16(a.bnd + 2 * (tile + 1), bnd_tag(epoch, BND_DONE), 0ull, succ_lo, succ_hi);
-        succ_pending = (succ_lo & 0xFFFFFFFFull) == bnd_tag(epoch, BND_PENDING);
-      } else {
-        succ_pending = (dev::atom_exch_acq_rel(a.bnd + 2 * (tile + 1), bnd_tag(epoch, BND_DONE)) & 0xFFFFFFFFull) ==
-                       bnd_tag(epoch, BND_PENDING);
-      }
-    }
-  }
+  if (t == C - 1) publish_carry<VT, H, EPI>(a, tile, epoch, Fall, hs, acc, Vex, succ_pending, succ_lo, succ_hi);
 
   // ---- step 2c/3b: combine and write back -----------------------------
   const bool dependent = hs && !Fex && tile > 0;  // the tile's first stop needs the carry
@@ -606,66 +700,193 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
     }
     return;
   }
-  // The warp holding the tile's first row stop needs the carry-in.  Non-blocking hand-off:
-  // if the predecessor has not published yet, leave the partial and its row behind and
-  // exchange the tile's hand-off word; whichever of the two tiles arrives second
-  // completes the segment (the other returns at once), so a tile never holds its SM
-  // slot waiting for a slower predecessor in the common case.  Same arithmetic either
-  // way: (fp64 partial + look-back fold) * inv, rounded once.
-  const unsigned dep_ballot = __ballot_sync(0xffffffffu, dependent);
-  if (dep_ballot) {
-    const int dep_lane = __ffs(dep_ballot) - 1;
-    unsigned long long sv = 0;
-    if (lane == 0) sv = dev::ld_relaxed(a.status + 2 * (tile - 1));
-    sv = __shfl_sync(0xffffffffu, sv, 0);
-    bool mine = true;
-    const bool can_pack = H > 1 || a.out_limit < (1ll << 32);  // h = 1 packs the row in 32 bits
-    if (((sv >> 2) != epoch || a.force_handoff) && can_pack) {  // predecessor still running: hand off
-      unsigned long long old = 0;
-      if (lane == dep_lane) {
-        if constexpr (H == 1) {
-          unsigned long long ohi;
-          dev::atom_exch_16(a.bnd + 2 * tile, ((unsigned long long)dep_row << 32) | bnd_tag(epoch, BND_PENDING),
-                            (unsigned long long)__double_as_longlong((double)dep[0]), old, ohi);
-        } else {
+  resolve_carries<VT, H, EPI>(a, out, tile, epoch, lane, wid, NW, dependent, dep, dep_row, inv, succ_pending,
+                              succ_lo, succ_hi);
+}
+
+// Strategy 2 (Fig. 10/12): no per-thread intermediate sums array.  The
+// first-result entries — stops before each thread in the tile, derived in-kernel
+// by a count scan instead of stored per thread — place every segment sum in a
+// per-workgroup result cache of RC = k*C entries in shared memory (k = result cache size,
+// Table 1); the thread walks its tile once, writing each completed segment straight
+// to its cache slot and keeping only the sum up to its first stop and its last partial
+// sum.  After the CTA scan the first stop's entry receives the scanned last partial sums
+// of the earlier threads, and the whole cache is written to y in a coalesced way.
+// Entries at or beyond RC ("more row stops than the result cache size") are complete
+// sums and go straight to y (the paper parks them in a global result array for a later
+// pass; on B200 the final value is already known).  The tile's first segment still
+// travels the cross-tile carry path of strategy 1 (thread 0's entry 0).
+template <typename VT, int H, int W, int T, int CM, int EPI>
+__device__ __forceinline__ void tile_body_s2(const KArgs& a, const int64_t tile, ScanShared<VT, H>& sh, VT* rcache) {
+  using TR = KTraits<VT, H, W, T, CM>;
+  constexpr int VB = TR::VB;
+  constexpr uint32_t TMASK = (T == 32) ? 0xffffffffu : ((1u << T) - 1u);
+  const int t = threadIdx.x, C = blockDim.x, lane = t & 31, wid = t >> 5, NW = C >> 5;
+  const int RC = a.rcache;
+  uint32_t fl;
+  uint32_t vw[H][VB / 4];
+  VT xs[T][W];
+  int cta_seg0;
+  unsigned long long tk = 0;
+  stream_tile<VT, H, W, T, CM, EPI>(a, tile, sh, t, C, fl, vw, xs, cta_seg0, tk);
+  VT* out = static_cast<VT*>(a.out);
+  const uint32_t stops = ~fl & TMASK;
+  const int nst = __popc(stops);
+  const int hs = nst > 0;
+
+  // first-result entries: inclusive count scan in the warp, warp totals through smem
+  int nin = nst;
 #pragma unroll
-          for (int r = 0; r < H; ++r) a.pend_val[tile * H + r] = (double)dep[r];
-          a.pend_row[tile] = dep_row;
-          old = dev::atom_exch_acq_rel(a.bnd + 2 * tile, bnd_tag(epoch, BND_PENDING));
+  for (int d = 1; d < 32; d <<= 1) {
+    const int n2 = __shfl_up_sync(0xffffffffu, nin, d);
+    if (lane >= d) nin += n2;
+  }
+  if (lane == 31) sh.wn[wid] = nin;
+  __syncthreads();
+  int Nw = 0, Ntot = 0;
+  for (int q = 0; q < NW; ++q) {
+    const int c = sh.wn[q];
+    if (q < wid) Nw += c;
+    Ntot += c;
+  }
+  const int fre = Nw + nin - nst;  // this thread's first stop, relative to the tile's first
+  const double inv = (EPI == 1 || EPI == 2) ? sh.inv : 1.0;
+  const VT invv = (VT)inv;
+  VT ssv = VT(0);
+  // a segment sum that is final: to its cache slot, or past the cache straight to y
+  auto emit = [&](const int e, const VT (&v)[H]) {
+    if (e < RC) {
+#pragma unroll
+      for (int r = 0; r < H; ++r) rcache[e * H + r] = v[r];
+    } else {
+      const int64_t row = a.seg_row ? (int64_t)__ldg(a.seg_row + cta_seg0 + e) : (int64_t)cta_seg0 + e;
+#pragma unroll
+      for (int r = 0; r < H; ++r)
+        if (row * H + r < a.out_limit) {
+          const VT o = (EPI == 1 || EPI == 2) ? v[r] * invv : v[r];
+          store_out<VT, EPI>(a, out, row * H + r, o);
+          if constexpr (EPI == 1 || EPI == 2) ssv = fma(o, o, ssv);
         }
-      }
-      old = __shfl_sync(0xffffffffu, old, dep_lane);
-      mine = (old & 0xFFFFFFFFull) == bnd_tag(epoch, BND_DONE);  // it published meanwhile: finish here
     }
-    if (mine) {
-      double carry[H];
-      lookback<H>(a, tile, epoch, lane, carry);
-      if (lane == dep_lane) {
-        double d[H];
+  };
+
+  // ---- multiply + sequential segmented sum straight into the result cache ----------
+  VT run[H], head[H];
 #pragma unroll
-        for (int r = 0; r < H; ++r) d[r] = (double)dep[r];
-        write_carried<VT, H, EPI>(a, out, tile, dep_row, d, carry, inv, NW);
+  for (int r = 0; r < H; ++r) run[r] = head[r] = VT(0);
+  int j = 0;
+#pragma unroll
+  for (int b = 0; b < T; ++b) {
+#pragma unroll
+    for (int r = 0; r < H; ++r) {
+      VT p = dev::word_val<VT>(vw[r], b * W) * xs[b][0];
+#pragma unroll
+      for (int c = 1; c < W; ++c) p = fma(dev::word_val<VT>(vw[r], b * W + c), xs[b][c], p);
+      run[r] = run[r] + p;
+    }
+    if ((stops >> b) & 1u) {
+      if (j == 0) {
+#pragma unroll
+        for (int r = 0; r < H; ++r) head[r] = run[r];
+      } else {
+        emit(fre + j, run);
       }
+      ++j;
+#pragma unroll
+      for (int r = 0; r < H; ++r) run[r] = VT(0);
     }
   }
-  // the next tile handed its carried segment to this one (its predecessor)
-  if (wid == NW - 1 && __shfl_sync(0xffffffffu, succ_pending ? 1 : 0, 31)) {
-    double carry[H];
-    lookback<H>(a, tile + 1, epoch, lane, carry);
-    if (lane == 31) {
-      double d[H];
-      int64_t row;
-      if constexpr (H == 1) {  // carried in the exchanged word
-        d[0] = __longlong_as_double((long long)succ_hi);
-        row = (int64_t)(succ_lo >> 32);
-      } else {  // lane 31's acquire (the exchange) made tile+1's pending data visible
+
+  // ---- CTA segmented scan of (has_stop, last partial sum) ----------
+  int f = hs;
+  VT v[H];
 #pragma unroll
-        for (int r = 0; r < H; ++r) d[r] = a.pend_val[(tile + 1) * H + r];
-        row = (int64_t)a.pend_row[tile + 1];
+  for (int r = 0; r < H; ++r) v[r] = run[r];
+  const unsigned hs_ballot = __ballot_sync(0xffffffffu, hs);
+  const bool warp_all_stop = (hs_ballot | 1u) == 0xffffffffu;  // skip
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int f2 = __shfl_up_sync(0xffffffffu, f, d);
+    if (!warp_all_stop) {
+#pragma unroll
+      for (int r = 0; r < H; ++r) {
+        const VT v2 = __shfl_up_sync(0xffffffffu, v[r], d);
+        if (lane >= d && !f) v[r] = v2 + v[r];
       }
-      write_carried<VT, H, EPI>(a, out, tile + 1, row, d, carry, inv, NW);
     }
+    if (lane >= d) f |= f2;
   }
+  if (lane == 31) {
+    sh.wf[wid] = f;
+#pragma unroll
+    for (int r = 0; r < H; ++r) sh.wv[wid][r] = v[r];
+  }
+  int fx = __shfl_up_sync(0xffffffffu, f, 1);
+  VT vx[H];
+#pragma unroll
+  for (int r = 0; r < H; ++r) vx[r] = __shfl_up_sync(0xffffffffu, v[r], 1);
+  if (lane == 0) {
+    fx = 0;
+#pragma unroll
+    for (int r = 0; r < H; ++r) vx[r] = VT(0);
+  }
+  if (a.block_ids && t == 0) sh.epoch = tk / (unsigned long long)a.period + 1ull;
+  __syncthreads();
+  const unsigned long long epoch = sh.epoch;
+  int Fw = 0, Fall = 0;
+  VT Vw[H];
+#pragma unroll
+  for (int r = 0; r < H; ++r) Vw[r] = VT(0);
+  for (int q = 0; q < NW; ++q) {
+    const int fq = sh.wf[q];
+    if (q < wid) {
+#pragma unroll
+      for (int r = 0; r < H; ++r) Vw[r] = fq ? sh.wv[q][r] : Vw[r] + sh.wv[q][r];
+      Fw |= fq;
+    }
+    Fall |= fq;
+  }
+  const int Fex = Fw | fx;
+  VT Vex[H];
+#pragma unroll
+  for (int r = 0; r < H; ++r) Vex[r] = fx ? vx[r] : Vw[r] + vx[r];
+
+  bool succ_pending = false;
+  unsigned long long succ_lo = 0, succ_hi = 0;
+  if (t == C - 1) publish_carry<VT, H, EPI>(a, tile, epoch, Fall, hs, run, Vex, succ_pending, succ_lo, succ_hi);
+
+  // ---- the first stop's entry gets the earlier threads' scanned partial sums --
+  const bool dependent = hs && !Fex && tile > 0;  // the tile's first segment: carry path
+  VT dep[H];
+  int64_t dep_row = 0;
+  if (hs) {
+#pragma unroll
+    for (int r = 0; r < H; ++r) dep[r] = head[r] + Vex[r];
+    if (dependent) dep_row = a.seg_row ? (int64_t)__ldg(a.seg_row + cta_seg0 + fre) : (int64_t)cta_seg0 + fre;
+    else emit(fre, dep);
+  }
+  __syncthreads();
+  // ---- coalesced write-back of the result cache (entry 0 of tiles > 0 is carried) ----
+  const int lim = min(Ntot, RC);
+  for (int e = (tile > 0 ? 1 : 0) + t; e < lim; e += C) {
+    const int64_t row = a.seg_row ? (int64_t)__ldg(a.seg_row + cta_seg0 + e) : (int64_t)cta_seg0 + e;
+#pragma unroll
+    for (int r = 0; r < H; ++r)
+      if (row * H + r < a.out_limit) {
+        const VT o = (EPI == 1 || EPI == 2) ? rcache[e * H + r] * invv : rcache[e * H + r];
+        store_out<VT, EPI>(a, out, row * H + r, o);
+        if constexpr (EPI == 1 || EPI == 2) ssv = fma(o, o, ssv);
+      }
+  }
+  if ((EPI == 1 || EPI == 2) && (a.epi & 2)) {  // per-warp partial of sum y^2, fixed tree (deterministic)
+    double ss = (double)ssv;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+    if (lane == 0) a.part[tile * (NW + 1) + wid] = ss;
+    if (t == 0 && !(Fall && tile > 0)) a.part[tile * (NW + 1) + NW] = 0.0;  // no carried segment
+  }
+  resolve_carries<VT, H, EPI>(a, out, tile, epoch, lane, wid, NW, dependent, dep, dep_row, inv, succ_pending,
+                              succ_lo, succ_hi);
 }
 
 // One CTA per workgroup-level tile; logical tile ids from an atomic ticket.
@@ -687,6 +908,29 @@ __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_kerne
   }
   __syncthreads();
   tile_body<VT, H, W, T, CM, EPI>(a, sh.tile, sh);
+}
+
+// Strategy-2 kernel (result cache in dynamic shared memory: KArgs::rcache entries of h values)
+template <typename VT, int H, int W, int T, int CM, int EPI>
+__global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_s2_kernel(const KArgs a) {
+  __shared__ ScanShared<VT, H> sh;
+  extern __shared__ __align__(16) unsigned char s2_rcache[];
+  VT* rcache = reinterpret_cast<VT*>(s2_rcache);
+  if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();
+  if (a.block_ids) {
+    tile_body_s2<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, sh, rcache);
+    return;
+  }
+  if (a.pdl) cudaGridDependencySynchronize();
+  if (threadIdx.x == 0) {
+    const unsigned long long tk = atomicAdd(a.ticket, 1ull);
+    const unsigned long long q = tk / (unsigned long long)a.period;
+    sh.tile = (long long)(tk - q * (unsigned long long)a.period);
+    sh.epoch = q + 1ull;
+    if constexpr (EPI == 1 || EPI == 2) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
+  }
+  __syncthreads();
+  tile_body_s2<VT, H, W, T, CM, EPI>(a, sh.tile, sh, rcache);
 }
 
 template <typename VT, int H, int W, int T, int CM>
@@ -713,7 +957,7 @@ void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
 }
 
 template <typename VT, int H, int W, int T, int CM>
-int attr_spmv(int C, int* regs, int* max_threads, int* blocks_per_sm) {
+int attr_spmv(int C, int /*rc*/, int* regs, int* max_threads, int* blocks_per_sm) {
   using TR = KTraits<VT, H, W, T, CM>;
   auto k = spmv_bccoo_kernel<VT, H, W, T, CM, 0>;
   auto k2 = spmv_bccoo_kernel<VT, H, W, T, CM, 1>;
@@ -749,13 +993,59 @@ int attr_spmv(int C, int* regs, int* max_threads, int* blocks_per_sm) {
   return 0;
 }
 
+template <typename VT, int H, int W, int T, int CM>
+void launch_spmv_s2(const KArgs& a, int C, int64_t grid, void* stream) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(C);
+  cfg.dynamicSmemBytes = (size_t)a.rcache * H * sizeof(VT);
+  cfg.stream = (cudaStream_t)stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (a.npeer > 0) cudaLaunchKernelEx(&cfg, spmv_bccoo_s2_kernel<VT, H, W, T, CM, 2>, a);
+  else if (a.epi) cudaLaunchKernelEx(&cfg, spmv_bccoo_s2_kernel<VT, H, W, T, CM, 1>, a);
+  else cudaLaunchKernelEx(&cfg, spmv_bccoo_s2_kernel<VT, H, W, T, CM, 0>, a);
+}
+
+template <typename VT, int H, int W, int T, int CM>
+int attr_spmv_s2(int C, int rc, int* regs, int* max_threads, int* blocks_per_sm) {
+  auto k0 = spmv_bccoo_s2_kernel<VT, H, W, T, CM, 0>;
+  auto k1 = spmv_bccoo_s2_kernel<VT, H, W, T, CM, 1>;
+  auto k2 = spmv_bccoo_s2_kernel<VT, H, W, T, CM, 2>;
+  cudaFuncAttributes fa;
+  cudaError_t e = cudaFuncGetAttributes(&fa, k0);
+  if (e != cudaSuccess) return (int)e;
+  *regs = fa.numRegs;
+  *max_threads = fa.maxThreadsPerBlock;
+  *blocks_per_sm = 0;
+  if (C > 0 && C <= *max_threads) {
+    const size_t dyn = (size_t)rc * C * H * sizeof(VT);
+    int optin = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    if (dyn + fa.sharedSizeBytes > (size_t)optin) return 0;
+    for (auto k : {k0, k1, k2}) {
+      e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+      if (e != cudaSuccess) return (int)e;
+      e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // the rest stays L1
+      if (e != cudaSuccess) return (int)e;
+    }
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k0, C, dyn);
+    if (e != cudaSuccess) return (int)e;
+  }
+  return 0;
+}
+
 template <typename VT, int H, int W, int T>
 void reg_t(std::vector<KernelEntry>& R) {
   if constexpr (T * H * W * (int)sizeof(VT) <= 512) {
     const int dt = sizeof(VT) == 4 ? 0 : 1;
-    R.push_back({dt, H, W, T, COL_U16, &launch_spmv<VT, H, W, T, COL_U16>, &attr_spmv<VT, H, W, T, COL_U16>});
-    R.push_back({dt, H, W, T, COL_I32, &launch_spmv<VT, H, W, T, COL_I32>, &attr_spmv<VT, H, W, T, COL_I32>});
-    R.push_back({dt, H, W, T, COL_DELTA, &launch_spmv<VT, H, W, T, COL_DELTA>, &attr_spmv<VT, H, W, T, COL_DELTA>});
+    R.push_back({dt, H, W, T, COL_U16, 1, &launch_spmv<VT, H, W, T, COL_U16>, &attr_spmv<VT, H, W, T, COL_U16>});
+    R.push_back({dt, H, W, T, COL_I32, 1, &launch_spmv<VT, H, W, T, COL_I32>, &attr_spmv<VT, H, W, T, COL_I32>});
+    R.push_back({dt, H, W, T, COL_DELTA, 1, &launch_spmv<VT, H, W, T, COL_DELTA>, &attr_spmv<VT, H, W, T, COL_DELTA>});
   }
 }
 
@@ -773,6 +1063,34 @@ void reg_h(std::vector<KernelEntry>& R) {
   reg_w<VT, H, 2>(R);
   reg_w<VT, H, 4>(R);
   reg_w<VT, H, 8>(R);
+}
+
+// strategy-2 instances (compiled in inst_s2_*.cu)
+template <typename VT, int H, int W, int T>
+void reg_t_s2(std::vector<KernelEntry>& R) {
+  if constexpr (T * H * W * (int)sizeof(VT) <= 512) {
+    const int dt = sizeof(VT) == 4 ? 0 : 1;
+    R.push_back({dt, H, W, T, COL_U16, 2, &launch_spmv_s2<VT, H, W, T, COL_U16>, &attr_spmv_s2<VT, H, W, T, COL_U16>});
+    R.push_back({dt, H, W, T, COL_I32, 2, &launch_spmv_s2<VT, H, W, T, COL_I32>, &attr_spmv_s2<VT, H, W, T, COL_I32>});
+    R.push_back(
+        {dt, H, W, T, COL_DELTA, 2, &launch_spmv_s2<VT, H, W, T, COL_DELTA>, &attr_spmv_s2<VT, H, W, T, COL_DELTA>});
+  }
+}
+
+template <typename VT, int H, int W>
+void reg_w_s2(std::vector<KernelEntry>& R) {
+  reg_t_s2<VT, H, W, 4>(R);
+  reg_t_s2<VT, H, W, 8>(R);
+  reg_t_s2<VT, H, W, 16>(R);
+  reg_t_s2<VT, H, W, 32>(R);
+}
+
+template <typename VT, int H>
+void reg_h_s2(std::vector<KernelEntry>& R) {
+  reg_w_s2<VT, H, 1>(R);
+  reg_w_s2<VT, H, 2>(R);
+  reg_w_s2<VT, H, 4>(R);
+  reg_w_s2<VT, H, 8>(R);
 }
 
 }  // namespace yaspmv

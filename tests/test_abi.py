@@ -62,3 +62,21 @@ def test_argument_errors():
         Matrix.from_csr(2, 70000, rp, c, v, device=-1, col_mode=1)       # u16 needs NB < 65535
     with pytest.raises(YaspmvError):
         Matrix.from_csr(2, 2, rp, c, v, device=-1, T=5)
+
+
+def test_result_cache_parameter():
+    """Table 1's strategy axis: result_cache 0 = strategy 1, {1,2,4} x C entries =
+    strategy 2; other values are refused; the resolved value round-trips through get_info."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix, YaspmvError
+    rp = np.array([0, 1, 2]); c = np.array([0, 1]); v = np.array([1.0, 2.0])
+    for rc in (0, 1, 2, 4):
+        A = Matrix.from_csr(2, 2, rp, c, v, device=-1, rc=rc)
+        assert A.info()["params"]["result_cache"] == rc
+        A.free()
+    A = Matrix.from_csr(2, 2, rp, c, v, device=-1, rc=-1)
+    assert A.info()["params"]["result_cache"] == 0
+    A.free()
+    for rc in (3, 5, 8):
+        with pytest.raises(YaspmvError) as e:
+            Matrix.from_csr(2, 2, rp, c, v, device=-1, rc=rc)
+        assert e.value.status == 1

@@ -142,3 +142,29 @@ def test_table3_dense_footprint():
                for h in (1, 2, 3, 4) for w in (1, 2, 4))
     assert round(best / 1e6) == g["bccoo_mb"]
     assert E.footprint_bytes(250_000, 4, 4, 4, 2) == best
+
+
+def test_strategy2_result_cache_fig10():
+    """O4 strategy 2 reproduces the Fig. 10 result-cache walk-through
+    on matrix C with R_i = 2^i, and its segment sums equal strategy 1's."""
+    g = load_golden("fig10_result_cache.txt")
+    gc = load_golden("fig6_matrix_C.txt")
+    bits = list(gc["flags"])
+    vals = [2 ** i for i in range(16)]
+    sums, trace = simulate.simulate_s2(vals, bits, 4, 4, 4)
+    tr = trace[0]
+    assert tr["fre"] == g["fre"]
+    assert tr["cache_walk"] == g["cache_walk"]
+    assert tr["cache"] == g["cache"]
+    assert sums == simulate.simulate(vals, bits, 4, 4)[0]
+
+
+@pytest.mark.parametrize("T,C,RC", [(4, 4, 1), (4, 4, 2), (2, 2, 2), (1, 16, 3), (8, 2, 1), (2, 4, 8)])
+def test_strategy2_equals_strategy1_across_workgroups(T, C, RC):
+    """Fig. 7 data over several workgroups with caches smaller than the stop count (the
+    global-result overflow of P:278) and larger: identical segment sums to strategy 1."""
+    g7 = load_golden("fig7_segscan.txt")
+    vals, bits = list(g7["input"]), list(g7["flags"])
+    pad = (-len(vals)) % (T * C)
+    s2, _ = simulate.simulate_s2(vals + [0] * pad, bits + [1] * pad, T, C, RC)
+    assert s2 == g7["segment_sums"]

@@ -53,7 +53,11 @@ def main():
     ap.add_argument("--iters", type=int, default=50)
     ap.add_argument("--md", default=None)
     ap.add_argument("--exhaustive", action="store_true", help="also run the exhaustive search (P:322)")
+    ap.add_argument("--from-jsonl", default=None, help="only rewrite --md from a previous run's JSON lines")
     args = ap.parse_args()
+    if args.from_jsonl:
+        write_md([json.loads(l) for l in open(args.from_jsonl) if l.startswith("{")], args.md)
+        return
     import torch
 
     import synth
@@ -93,7 +97,8 @@ def main():
         # the same tuned parameters launched without programmatic dependent launch
         q = {k: v for k, v in chosen.items()}
         B = Matrix.from_synth(csr, device=0, h=q["block_h"], w=q["block_w"], S=q["slices"], T=q["thread_tile"],
-                              C=q["cta_size"], col_mode=q["col_mode"], empty_mode=q["empty_mode"], flags=16)
+                              C=q["cta_size"], col_mode=q["col_mode"], empty_mode=q["empty_mode"],
+                              rc=q.get("result_cache", 0), flags=16)
         b2b_nopdl = timed_b2b(lambda: B.spmv(x, y))
         B.free()
         r = {"config": name, "m": csr.m, "nnz": csr.nnz, "dtype": str(dt), "params": chosen,
@@ -108,25 +113,30 @@ def main():
         rows.append(r)
         A.free()
     if args.md:
-        with open(args.md, "w") as f:
-            f.write("| config | nnz | dtype | tuned (h,w,T,C,S,col) | tune s | warm ms | cold ms | back-to-back ms (no PDL) | GFLOPS (cold) | alg GB/s (cold) | frac of measured HBM | parity (worst err/tol) | oracle CPU ms |\n")
-            f.write("|---|---|---|---|---|---|---|---|---|---|---|---|---|\n")
+        write_md(rows, args.md)
+
+
+
+def write_md(rows, path):
+    with open(path, "w") as f:
+        f.write("| config | nnz | dtype | tuned (h,w,T,C,S,col,rc) | tune s | warm ms | cold ms | back-to-back ms (no PDL) | GFLOPS (cold) | alg GB/s (cold) | frac of measured HBM | parity (worst err/tol) | oracle CPU ms |\n")
+        f.write("|---|---|---|---|---|---|---|---|---|---|---|---|---|\n")
+        for r in rows:
+            p = r["params"]
+            f.write(f"| {r['config']} | {r['nnz']:,} | {r['dtype']} | {p['block_h']}x{p['block_w']}, T={p['thread_tile']}, "
+                    f"C={p['cta_size']}, S={p['slices']}, col={p['col_mode']}, rc={p.get('result_cache', 0)} | {r['tune_s']:.1f} | {r['ms_warm']:.4f} | "
+                    f"{r['ms_cold']:.4f} | {r['ms_b2b']:.4f} ({r['ms_b2b_no_pdl']:.4f}) | {r['gflops_cold']:.1f} | {r['alg_GBs_cold']:.0f} | {r['frac_of_measured_hbm_cold']:.3f} | "
+                    f"{'ok' if r['parity_ok'] else 'FAIL'} ({r['worst_err_over_tol']:.2g}) | {r['oracle_cpu_ms']:.2f} |\n")
+        if any(r["exhaustive"] for r in rows):
+            f.write("\n### tuned (4 smallest-footprint shapes, P:321) vs exhaustive over all compiled shapes (P:322)\n\n")
+            f.write("| config | tuned params | tuned warm ms | exhaustive params | exhaustive warm ms | exhaustive tune s | tuned/exhaustive time |\n|---|---|---|---|---|---|---|\n")
             for r in rows:
-                p = r["params"]
-                f.write(f"| {r['config']} | {r['nnz']:,} | {r['dtype']} | {p['block_h']}x{p['block_w']}, T={p['thread_tile']}, "
-                        f"C={p['cta_size']}, S={p['slices']}, col={p['col_mode']} | {r['tune_s']:.1f} | {r['ms_warm']:.4f} | "
-                        f"{r['ms_cold']:.4f} | {r['ms_b2b']:.4f} ({r['ms_b2b_no_pdl']:.4f}) | {r['gflops_cold']:.1f} | {r['alg_GBs_cold']:.0f} | {r['frac_of_measured_hbm_cold']:.3f} | "
-                        f"{'ok' if r['parity_ok'] else 'FAIL'} ({r['worst_err_over_tol']:.2g}) | {r['oracle_cpu_ms']:.2f} |\n")
-            if any(r["exhaustive"] for r in rows):
-                f.write("\n### tuned (4 smallest-footprint shapes, P:321) vs exhaustive over all compiled shapes (P:322)\n\n")
-                f.write("| config | tuned params | tuned warm ms | exhaustive params | exhaustive warm ms | exhaustive tune s | tuned/exhaustive time |\n|---|---|---|---|---|---|---|\n")
-                for r in rows:
-                    e = r["exhaustive"]
-                    if not e:
-                        continue
-                    p, q = r["params"], e["params"]
-                    f.write(f"| {r['config']} | {p['block_h']}x{p['block_w']} T={p['thread_tile']} C={p['cta_size']} | {r['ms_warm']:.4f} | "
-                            f"{q['block_h']}x{q['block_w']} T={q['thread_tile']} C={q['cta_size']} | {e['ms_warm']:.4f} | {e['tune_s']:.1f} | {r['ms_warm'] / e['ms_warm']:.3f} |\n")
+                e = r["exhaustive"]
+                if not e:
+                    continue
+                p, q = r["params"], e["params"]
+                f.write(f"| {r['config']} | {p['block_h']}x{p['block_w']} T={p['thread_tile']} C={p['cta_size']} | {r['ms_warm']:.4f} | "
+                        f"{q['block_h']}x{q['block_w']} T={q['thread_tile']} C={q['cta_size']} | {e['ms_warm']:.4f} | {e['tune_s']:.1f} | {r['ms_warm'] / e['ms_warm']:.3f} |\n")
 
 
 if __name__ == "__main__":
