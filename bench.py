@@ -211,7 +211,7 @@ def main():
     ap.add_argument("--config", default="c5")
     ap.add_argument("--params", default=None, help="JSON dict of build parameters")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=20)
+    ap.add_argument("--e2e-steps", type=int, default=30)
     ap.add_argument("--backend", default="nccl", help="process-group backend for N > 1 (gloo: exchange-path "
                     "check with several ranks on one GPU; never a performance number)")
     ap.add_argument("--rows", type=int, default=0, help="C5 only: use the first ROWS rows/cols (checks)")
@@ -346,7 +346,7 @@ def main():
 
     # ---- e2e through the public API with HOST buffers (pinned) -----------------------
     # every step copies x host->device and y device->host; yaspmv_spmv_host_async overlaps
-    # the copies of consecutive steps with the SpMV (two buffer slots, two copy streams)
+    # the copies of consecutive steps with the SpMV (three buffer slots, two copy streams)
     xh = torch.empty(L.n_padded, dtype=tdt).pin_memory()
     x_cur = fpit.current_x(stream) if fpit is not None else pit.current_x()
     xh.copy_(x_cur.cpu())

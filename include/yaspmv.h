@@ -81,6 +81,12 @@ typedef struct {
                            P:293).  Results agree within rounding (the first stop's sum is
                            associated differently).  yaspmv_reencode: 0 = keep current,
                            -1 = strategy 1.  A launch-time choice: no re-encode needed. */
+  int32_t tiles_per_cta; /* consecutive workgroup-level tiles one CTA processes (B200
+                           scheduling, not in Table 1): 0 = auto (2 when the matrix has
+                           >= 32 waves of tiles, else 1), k in 1..64.  A warp that finishes
+                           a tile issues the next tile's loads at once while the tile's
+                           stores drain.  Results are bitwise identical for every k.
+                           Launch-time (no re-encode); forced to 1 with YASPMV_TICKET_IDS. */
 } yaspmv_params;
 
 typedef struct {
@@ -164,7 +170,8 @@ yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host
 
 /* yaspmv_spmv_host_async: y := A·x with HOST x / y, returning before completion.  Calls on
  * one handle overlap the host->device copy of call k+1, the SpMV of call k and the
- * device->host copy of call k-1 (two handle-owned device buffer pairs, two internal copy
+ * device->host copy of call k-1 (three handle-owned device buffer pairs — with two, the
+ * copy-in of call k would wait for the copy-out of call k-2 — two internal copy
  * streams, events chaining them to `stream`).  x_host must stay unchanged and y_host valid
  * until yaspmv_host_sync(A); pinned host memory is needed for the copies to overlap.
  * yaspmv_host_sync: waits for every outstanding yaspmv_spmv_host_async of the handle. */
@@ -175,8 +182,8 @@ yaspmv_status yaspmv_host_sync(yaspmv_matrix A);
  * yaspmv_tune: auto-tuner of PAPER.md §4: for the 4 block shapes with the
  * smallest footprint it times the SpMV over thread tile T, CTA size C, slice count
  * S and column mode with strategy 1, then strategy 2 with result cache sizes 1 and 2 (the
- * paper's pinned values) for the two fastest (T, C) of each (h, w, S, col mode), on
- * the device (scratch x/y owned by the tuner), then re-encodes A with
+ * paper's pinned values) for every (T, C), then tiles_per_cta in {1, 2, 4} for the
+ * winner, on the device (scratch x/y owned by the tuner), then re-encodes A with
  * the fastest parameters (ties within 1%: smaller footprint, then lexicographic).
  * Re-encoding needs the normalised CSR the handle keeps unless built with
  * YASPMV_DROP_CSR (then EINVAL).  On failure A keeps its previous parameters.
@@ -188,7 +195,8 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen);
 yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode);
 
 /* yaspmv_reencode: re-encode A with new parameters (0 fields = keep current; see
- * result_cache for its -1).  A change of result_cache alone only re-selects the kernel. */
+ * result_cache for its -1).  A change of result_cache / tiles_per_cta alone only
+ * re-selects the launch (no re-encode). */
 yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params);
 
 /* ---------------------------------------------------------------- introspection

@@ -41,7 +41,8 @@ EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv"
 class Params(ctypes.Structure):
     _fields_ = [("block_h", ctypes.c_int32), ("block_w", ctypes.c_int32), ("slices", ctypes.c_int32),
                 ("thread_tile", ctypes.c_int32), ("cta_size", ctypes.c_int32), ("col_mode", ctypes.c_int32),
-                ("empty_mode", ctypes.c_int32), ("flags", ctypes.c_int32), ("result_cache", ctypes.c_int32)]
+                ("empty_mode", ctypes.c_int32), ("flags", ctypes.c_int32), ("result_cache", ctypes.c_int32),
+                ("tiles_per_cta", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}

@@ -56,6 +56,7 @@ Params from_abi(const yaspmv_params* p) {
     q.empty_mode = p->empty_mode;
     q.flags = p->flags;
     q.rc = p->result_cache;
+    q.tpc = p->tiles_per_cta;
   }
   return q;
 }
@@ -71,6 +72,7 @@ yaspmv_params to_abi(const Params& q) {
   p.empty_mode = q.empty_mode;
   p.flags = q.flags;
   p.result_cache = q.rc;
+  p.tiles_per_cta = q.tpc;
   return p;
 }
 
@@ -175,9 +177,12 @@ yaspmv_status select_kernel(yaspmv_matrix A) {
   if (bps <= 0) return fail(YASPMV_EUNSUPPORTED, "kernel does not fit on an SM with this cta_size");
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, A->device);
-  // one CTA per workgroup-level tile (ticketed)
-  A->grid = std::max<int64_t>(1, A->can.ntiles);
-  (void)sms;
+  // one CTA per tiles_per_cta consecutive workgroup-level tiles; auto: 2 once the
+  // matrix spans >= 32 waves of resident CTAs (C5: 244,680 tiles; measured 4.17 vs 4.52 ms)
+  if (p.tpc > 0) A->tpc = p.tpc;
+  else A->tpc = A->can.ntiles >= 32LL * std::max(1, sms) * bps ? 2 : 1;
+  if (p.flags & YASPMV_TICKET_IDS) A->tpc = 1;
+  A->grid = std::max<int64_t>(1, (A->can.ntiles + A->tpc - 1) / A->tpc);
   A->regs = regs;
   return YASPMV_OK;
 }
@@ -374,6 +379,7 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   a.npeer = 0;
   for (int q = 0; q < YASPMV_MAX_RANKS; ++q) a.peer_out[q] = nullptr;
   a.rcache = p.rc * p.C;
+  a.tpc = A->tpc;
   if (ablate && p.rc > 0) return fail(YASPMV_EUNSUPPORTED, "ablation / probe variants are strategy-1 kernels");
   if (peers && p.S == 1) {  // S > 1: the kernel writes tmp, the combine writes the peers
     a.npeer = peers->n;
@@ -411,17 +417,20 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
 
 }  // namespace
 
-// switch the segmented-sum strategy of an encoded handle (kernel re-selection only)
-yaspmv_status set_strategy(yaspmv_matrix A, int rc) {
-  const int old = A->can.p.rc;
+// switch the launch-time parameters (strategy, tiles per CTA) of an encoded handle
+yaspmv_status set_launch(yaspmv_matrix A, int rc, int tpc) {
+  const int orc = A->can.p.rc, otpc = A->can.p.tpc, oldt = A->tpc;
   const KernelEntry* oldk = A->kern;
   const int64_t oldgrid = A->grid;
   A->can.p.rc = rc;
+  A->can.p.tpc = tpc;
   yaspmv_status st = select_kernel(A);
   if (st != YASPMV_OK) {
-    A->can.p.rc = old;
+    A->can.p.rc = orc;
+    A->can.p.tpc = otpc;
     A->kern = oldk;
     A->grid = oldgrid;
+    A->tpc = oldt;
   }
   return st;
 }
@@ -491,14 +500,17 @@ yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
   if (!want.S) want.S = cur.S;
   if (!want.T) want.T = cur.T;
   if (!want.C) want.C = cur.C;
+  if (!want.col_mode) want.col_mode = cur.col_mode;
+  if (!want.empty_mode) want.empty_mode = cur.empty_mode;
   if (!params) want.flags = cur.flags;
   want.rc = want.rc == 0 ? cur.rc : (want.rc < 0 ? 0 : want.rc);
-  {  // only the strategy changes: a launch-time choice, no re-encode (Table 1 axes T..S unchanged)
+  if (!want.tpc) want.tpc = cur.tpc;
+  {  // only launch-time parameters change (strategy, tiles per CTA): no re-encode
     Params rp;
     if (A->device >= 0 && resolve_params(want, A->csr.m, A->csr.n, rp) == YASPMV_OK && rp.h == cur.h &&
         rp.w == cur.w && rp.S == cur.S && rp.T == cur.T && rp.C == cur.C && rp.col_mode == cur.col_mode &&
         (rp.empty_mode == 0 || rp.empty_mode == cur.empty_mode) && rp.flags == cur.flags)
-      return set_strategy(A, rp.rc);
+      return set_launch(A, rp.rc, rp.tpc);
   }
   return encode_into(A, want);
 }
@@ -566,7 +578,7 @@ yaspmv_status yaspmv_spmv_host_async(yaspmv_matrix A, const void* x_host, void* 
     }
   }
   auto& s = A->hslot[A->next_slot];
-  A->next_slot ^= 1;
+  A->next_slot = (A->next_slot + 1) % 3;
   cudaStream_t cs = (cudaStream_t)stream;
   CUDA_TRY(cudaStreamWaitEvent(A->s_in, s.done, 0));  // the slot's previous copy-out is done
   if (xb) CUDA_TRY(cudaMemcpyAsync(s.x, x_host, xb, cudaMemcpyHostToDevice, A->s_in));
@@ -599,7 +611,7 @@ int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
 yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle");
-  if (variant < 1 || variant > 9) return fail(YASPMV_EINVAL, "ablation variant must be in 1..9");
+  if (variant < 1 || variant > 11) return fail(YASPMV_EINVAL, "ablation variant must be in 1..11");
   if (variant != 3 && (A->can.p.h != 1 || A->can.p.w != 1))
     return fail(YASPMV_EUNSUPPORTED, "ablation variants / probes are compiled for 1x1 blocks only");
   const int ab = variant == 1   ? ABL_DEFER_CARRY
@@ -610,7 +622,9 @@ yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void*
                  : variant == 7 ? (ABL_DEFER_CARRY | ABL_NO_FIXUP)
                  : variant == 8 ? ABL_STOP_SCAN
                  : variant == 9 ? (ABL_DEFER_CARRY | ABL_NO_FIXUP | ABL_NO_YSTORE)
-                                : 0;
+                 : variant == 10 ? (ABL_STOP_SCAN | ABL_PROBE_PUB)
+                 : variant == 11 ? (ABL_STOP_SCAN | ABL_PROBE_ST)
+                                 : 0;
   return run_spmv(A, x, y, stream, nullptr, nullptr, ab);
 }
 
@@ -658,6 +672,7 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
   o->alg_bytes = alg_bytes(A);
   o->footprint_bytes = footprint_bytes(c.nnzb, c.p.h, c.p.w, A->vsize, col_bytes(c.p.col_mode));
   o->params = to_abi(c.p);
+  if (A->device >= 0) o->params.tiles_per_cta = A->tpc;  // the resolved value
   o->dtype = A->dtype;
   o->device = A->device;
   o->has_seg_row = c.has_seg_row;

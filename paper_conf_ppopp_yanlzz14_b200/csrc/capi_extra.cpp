@@ -220,6 +220,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
 
   struct Cand { float ms; int64_t bytes; Params p; };
   std::vector<Cand> results;
+  int results_extra = 0;
   const Params saved = A->can.p;
   const int keep_flags = saved.flags & ~YASPMV_DROP_CSR;
   for (const Shape& sh : shapes) {
@@ -235,6 +236,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
         Params bp0;
         bp0.h = sh.h; bp0.w = sh.w; bp0.S = S; bp0.T = 32; bp0.C = 512; bp0.col_mode = cm;
         bp0.empty_mode = saved.empty_mode;
+        bp0.tpc = 1;
         Params rp;
         if (resolve_params(bp0, M.m, M.n, rp) != YASPMV_OK) continue;
         Canonical base;
@@ -247,7 +249,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             const int64_t tiles = (nnzb_est + (int64_t)T * C - 1) / ((int64_t)T * C);
             if (tiles < 2 * sms && (T * C) > 1024) continue;
             if (gpu) {
-              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode, YASPMV_GPU_ENCODE, -1};
+              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode, YASPMV_GPU_ENCODE, -1, 1};
               if (yaspmv_reencode(A, &ap) != YASPMV_OK) continue;
             } else {
               Canonical cand;
@@ -274,7 +276,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             // strategy 2 with the paper's pinned result cache sizes 1 and 2: a
             // launch-time switch on the same encoding
             for (int rc : {1, 2}) {
-              if (!find_kernel(A->dtype, sh.h, sh.w, T, cm, 2) || set_strategy(A, rc) != YASPMV_OK) continue;
+              if (!find_kernel(A->dtype, sh.h, sh.w, T, cm, 2) || set_launch(A, rc, 1) != YASPMV_OK) continue;
               bool ok2 = true;
               for (int it = 0; it < 3 && ok2; ++it) ok2 = yaspmv_spmv(A, x, y, stream) == YASPMV_OK;
               if (ok2) {
@@ -291,20 +293,23 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
                 std::sort(t2.begin(), t2.end());
                 results.push_back({t2[t2.size() / 2], info.format_bytes, A->can.p});
               }
-              set_strategy(A, 0);
+              set_launch(A, 0, 1);
             }
           }
         }
       }
     }
   }
-  cudaEventDestroy(e0);
-  cudaEventDestroy(e1);
-  cudaFree(x);
-  cudaFree(y);
+  auto release = [&]() {
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(x);
+    cudaFree(y);
+  };
   if (results.empty()) {
+    release();
     yaspmv_params back{saved.h, saved.w, saved.S, saved.T, saved.C, saved.col_mode, saved.empty_mode, keep_flags,
-                       saved.rc > 0 ? saved.rc : -1};
+                       saved.rc > 0 ? saved.rc : -1, saved.tpc};
     yaspmv_reencode(A, &back);
     return fail(YASPMV_EUNSUPPORTED, "no tunable candidate could be launched");
   }
@@ -319,14 +324,46 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
     if (key(c) < key(*best)) best = &c;
   }
   yaspmv_params bp{best->p.h, best->p.w, best->p.S, best->p.T, best->p.C, best->p.col_mode, best->p.empty_mode,
-                   keep_flags, best->p.rc > 0 ? best->p.rc : -1};
+                   keep_flags, best->p.rc > 0 ? best->p.rc : -1, 1};
   yaspmv_status rs = yaspmv_reencode(A, &bp);
-  if (rs != YASPMV_OK) return rs;
+  if (rs != YASPMV_OK) {
+    release();
+    return rs;
+  }
+  // (4) tiles per CTA for the winner (launch-time; bitwise-identical results): fastest,
+  // ties within 1% to the smaller count
+  {
+    float tbest = 1e30f;
+    int kbest = 1;
+    for (int k : {1, 2, 4}) {
+      if (set_launch(A, A->can.p.rc, k) != YASPMV_OK) continue;
+      for (int it = 0; it < 3; ++it) yaspmv_spmv(A, x, y, stream);
+      std::vector<float> tk;
+      for (int it = 0; it < 7; ++it) {
+        cudaEventRecord(e0, st);
+        yaspmv_spmv(A, x, y, stream);
+        cudaEventRecord(e1, st);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        tk.push_back(ms);
+      }
+      std::sort(tk.begin(), tk.end());
+      const float med = tk[tk.size() / 2];
+      if (med < tbest * 0.99f) {
+        tbest = med;
+        kbest = k;
+      }
+      ++results_extra;
+    }
+    set_launch(A, A->can.p.rc, kbest);
+  }
+  release();
   A->tune_s = now_s() - t0;
-  A->tune_candidates = (int)results.size();
+  A->tune_candidates = (int)results.size() + results_extra;
   if (chosen) {
     const Params& q = A->can.p;
-    *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags, q.rc};
+    *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags, q.rc, A->tpc};
   }
   return YASPMV_OK;
 }

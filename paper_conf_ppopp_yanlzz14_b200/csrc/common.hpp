@@ -24,12 +24,17 @@ enum Ablate {
   ABL_GATHER_L2 = 16,  // with GATHER_ONLY: gathers of x[col & (2^20-1)] (4-8 MB: L2 hits, L1 misses)
   ABL_STOP_SCAN = 32,  // probe: return right after the CTA scan (no publish, stores, carries)
   ABL_NO_FIXUP = 64,  // host side, with DEFER_CARRY: no carry kernel ("no carries" probe)
-  ABL_NO_YSTORE = 256  // probe: y stores of the FILLER write-back skipped
+  ABL_NO_YSTORE = 256,  // probe: y stores of the FILLER write-back skipped
+  // with STOP_SCAN: after the scan, thread C-1 stores the tile's status word (PUB) / every
+  // thread stores one value, coalesced (ST) — the cost of a CTA ending in stores
+  ABL_PROBE_PUB = 512,
+  ABL_PROBE_ST = 1024
 };
 
 struct Params {
   int h = 1, w = 1, S = 1, T = 16, C = 256, col_mode = 0, empty_mode = 0, flags = 0;
   int rc = 0;  // result cache size in units of C: 0 = strategy 1, k > 0 = strategy 2 (Table 1)
+  int tpc = 0;  // tiles per CTA (0 = auto)
 };
 
 inline int col_bytes(int mode) { return mode == COL_I32 ? 4 : 2; }
@@ -154,6 +159,7 @@ struct KArgs {
   int npeer;
   void* peer_out[YASPMV_MAX_RANKS];
   int rcache;              // strategy 2: result cache entries (rc * C); 0 for strategy 1
+  int tpc;                 // consecutive tiles per workgroup (block-id mode); grid = ceil(ntiles / tpc)
 };
 
 // destinations of a fused exchange (combine kernel of BCCOO+, S > 1)

@@ -196,6 +196,7 @@ yaspmv_status resolve_params(const Params& in, int64_t m, int64_t n, Params& out
   if (out.rc < 0) out.rc = 0;  // -1 = strategy 1 explicitly (yaspmv_reencode)
   if (out.rc != 0 && out.rc != 1 && out.rc != 2 && out.rc != 4)
     return fail(YASPMV_EINVAL, "result_cache must be 0 (strategy 1) or 1, 2, 4 (x C entries, strategy 2)");
+  if (out.tpc < 0 || out.tpc > 64) return fail(YASPMV_EINVAL, "tiles_per_cta must be 0 (auto) or in 1..64");
   (void)m;
   return YASPMV_OK;
 }

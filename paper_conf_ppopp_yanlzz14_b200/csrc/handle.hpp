@@ -44,15 +44,17 @@ struct yaspmv_matrix_s {
   DevArrays d;
   const KernelEntry* kern = nullptr;
   int regs = 0;
-  int64_t grid = 1;  // persistent CTAs per launch (fixed per encoding: ticket period)
+  int64_t grid = 1;  // CTAs per launch
+  int tpc = 1;       // resolved tiles per CTA (params.tiles_per_cta; block-id mode only)
   void* xs = nullptr;  // scratch for spmv_host
   void* ys = nullptr;
-  // spmv_host_async: two buffer slots, two copy streams, chaining events
+  // spmv_host_async: three buffer slots (H2D of call k+1, SpMV of call k and D2H of call k-1
+  // in flight with no slot reuse stalling the pipeline), two copy streams, chaining events
   struct HostSlot {
     void* x = nullptr;
     void* y = nullptr;
     cudaEvent_t in = nullptr, comp = nullptr, done = nullptr;
-  } hslot[2];
+  } hslot[3];
   cudaStream_t s_in = nullptr, s_out = nullptr;
   int next_slot = 0;
   double* d_part = nullptr;     // power-iteration epilogue: partials of sum y^2
@@ -95,5 +97,6 @@ yaspmv_status install_canonical(yaspmv_matrix A, Canonical&& c, int flags);
 // of a local y (the fused exchange of comm.cu); out_norm2 receives sum y^2 (nullable)
 yaspmv_status run_spmv_peers(yaspmv_matrix A, const void* x, const double* in_norm2, double* out_norm2,
                              const yaspmv::PeerOut& peers, void* stream);
-// capi.cpp: switch the segmented-sum strategy (result_cache) of an encoded handle
-yaspmv_status set_strategy(yaspmv_matrix A, int rc);
+// capi.cpp: switch the launch-time parameters (result_cache, tiles_per_cta; 0 = auto) of an
+// encoded handle
+yaspmv_status set_launch(yaspmv_matrix A, int rc, int tpc);

@@ -1,8 +1,8 @@
-// Precompiled strategy-2 (per-workgroup result cache) SpMV kernel instances: dtype double, block
+// Precompiled strategy-1 (intermediate sums in registers) SpMV kernel instances: dtype float, block
 // height 4, block widths {1,2,4,8} x thread tiles {4,8,16,32} x column modes (Table 1,
 // P:305-319), restricted to T*h*w*sizeof(value) <= 512 bytes of values per thread.
 #include "spmv_kernel.cuh"
 
 namespace yaspmv {
-void register_s2_f64_h4(std::vector<KernelEntry>& R) { reg_h_s2<double, 4>(R); }
+void register_s1_f32_h4(std::vector<KernelEntry>& R) { reg_h<float, 4>(R); }
 }  // namespace yaspmv

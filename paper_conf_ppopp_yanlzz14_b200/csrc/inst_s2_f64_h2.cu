@@ -1,6 +1,6 @@
-// Precompiled strategy-2 SpMV kernel instances (result cache, Table 1):
-// dtype double, block height 2, block widths {1,2,4,8} x thread tiles {4,8,16,32} x column
-// modes, restricted to T*h*w*sizeof(value) <= 512 bytes of values per thread.
+// Precompiled strategy-2 (per-workgroup result cache) SpMV kernel instances: dtype double, block
+// height 2, block widths {1,2,4,8} x thread tiles {4,8,16,32} x column modes (Table 1,
+// P:305-319), restricted to T*h*w*sizeof(value) <= 512 bytes of values per thread.
 #include "spmv_kernel.cuh"
 
 namespace yaspmv {

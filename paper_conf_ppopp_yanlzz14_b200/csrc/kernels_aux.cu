@@ -161,14 +161,14 @@ void launch_scale(const void* src, void* dst, int64_t n, int dtype, const double
 }
 
 // ---------------------------------------------------------------- registry
-void register_f32_h1(std::vector<KernelEntry>&);
-void register_f32_h2(std::vector<KernelEntry>&);
-void register_f32_h3(std::vector<KernelEntry>&);
-void register_f32_h4(std::vector<KernelEntry>&);
-void register_f64_h1(std::vector<KernelEntry>&);
-void register_f64_h2(std::vector<KernelEntry>&);
-void register_f64_h3(std::vector<KernelEntry>&);
-void register_f64_h4(std::vector<KernelEntry>&);
+void register_s1_f32_h1(std::vector<KernelEntry>&);
+void register_s1_f32_h2(std::vector<KernelEntry>&);
+void register_s1_f32_h3(std::vector<KernelEntry>&);
+void register_s1_f32_h4(std::vector<KernelEntry>&);
+void register_s1_f64_h1(std::vector<KernelEntry>&);
+void register_s1_f64_h2(std::vector<KernelEntry>&);
+void register_s1_f64_h3(std::vector<KernelEntry>&);
+void register_s1_f64_h4(std::vector<KernelEntry>&);
 void register_s2_f32_h1(std::vector<KernelEntry>&);
 void register_s2_f32_h2(std::vector<KernelEntry>&);
 void register_s2_f32_h3(std::vector<KernelEntry>&);
@@ -182,14 +182,14 @@ const std::vector<KernelEntry>& all_kernels() {
   static std::vector<KernelEntry> R;
   static std::once_flag once;
   std::call_once(once, [] {
-    register_f32_h1(R);
-    register_f32_h2(R);
-    register_f32_h3(R);
-    register_f32_h4(R);
-    register_f64_h1(R);
-    register_f64_h2(R);
-    register_f64_h3(R);
-    register_f64_h4(R);
+    register_s1_f32_h1(R);
+    register_s1_f32_h2(R);
+    register_s1_f32_h3(R);
+    register_s1_f32_h4(R);
+    register_s1_f64_h1(R);
+    register_s1_f64_h2(R);
+    register_s1_f64_h3(R);
+    register_s1_f64_h4(R);
     register_s2_f32_h1(R);
     register_s2_f32_h2(R);
     register_s2_f32_h3(R);

@@ -593,7 +593,15 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
 #pragma unroll
   for (int r = 0; r < H; ++r) Vex[r] = fx ? vx[r] : Vw[r] + vx[r];
   if (EPI == 3 && (a.ablate & ABL_STOP_SCAN)) {  // roofline probe: everything up to the scan
-    if (Vex[0] == VT(-1.25e-30) || Nex == -7) out[t] = Vex[0];
+    if (a.ablate & ABL_PROBE_PUB) {
+      if (t == C - 1)
+        dev::st_relaxed_16(a.status + 2 * tile, (epoch << 2) | (Fall ? 2ull : 1ull),
+                           (unsigned long long)__double_as_longlong((double)Vex[0]));
+    } else if (a.ablate & ABL_PROBE_ST) {
+      out[(tile * C + t) % a.out_limit] = Vex[0] + VT(Nex);
+    } else if (Vex[0] == VT(-1.25e-30) || Nex == -7) {
+      out[t] = Vex[0];
+    }
     return;
   }
 
@@ -892,10 +900,21 @@ __device__ __forceinline__ void tile_body_s2(const KArgs& a, const int64_t tile,
 // One CTA per workgroup-level tile; logical tile ids from an atomic ticket.
 template <typename VT, int H, int W, int T, int CM, int EPI>
 __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_kernel(const KArgs a) {
-  __shared__ ScanShared<VT, H> sh;
+  __shared__ ScanShared<VT, H> shb[2];
+  ScanShared<VT, H>& sh = shb[0];
   if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();  // the next SpMV may start its loads
   if (a.block_ids) {  // tile = workgroup id: workgroups dispatch in order — the default
-    tile_body<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, sh);
+    if (a.tpc <= 1) {
+      tile_body<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, sh);
+      return;
+    }
+    // tpc consecutive tiles per workgroup: a warp done with one tile issues the next
+    // tile's loads at once (no barrier between tiles) while the tile's stores drain and its
+    // look-back completes.  The scan state alternates between two buffers: the scan barrier
+    // of tile k+1 is passed only when every warp has finished tile k, so tile k+2 can
+    // reuse tile k's buffer.
+    const int64_t t0 = (int64_t)blockIdx.x * a.tpc, t1 = min(a.ntiles, t0 + a.tpc);
+    for (int64_t tile = t0; tile < t1; ++tile) tile_body<VT, H, W, T, CM, EPI>(a, tile, shb[tile & 1]);
     return;
   }
   if (a.pdl) cudaGridDependencySynchronize();
@@ -918,7 +937,12 @@ __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_s2_ke
   VT* rcache = reinterpret_cast<VT*>(s2_rcache);
   if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();
   if (a.block_ids) {
-    tile_body_s2<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, sh, rcache);
+    // consecutive tiles without a barrier in between: each state (counts, scan values,
+    // result cache) is written in tile k+1 only after a barrier that every warp reaches
+    // after its last read of that state in tile k (count scan -> B1, walk -> B2, cache
+    // write-back -> next tile's B1)
+    const int64_t t0 = (int64_t)blockIdx.x * max(a.tpc, 1), t1 = min(a.ntiles, t0 + max(a.tpc, 1));
+    for (int64_t tile = t0; tile < t1; ++tile) tile_body_s2<VT, H, W, T, CM, EPI>(a, tile, sh, rcache);
     return;
   }
   if (a.pdl) cudaGridDependencySynchronize();

@@ -37,7 +37,7 @@ def _stream(stream) -> int | None:
 def make_params(**kw) -> _lib.Params:
     p = _lib.Params()
     names = {"h": "block_h", "w": "block_w", "S": "slices", "T": "thread_tile", "C": "cta_size",
-             "rc": "result_cache"}
+             "rc": "result_cache", "tpc": "tiles_per_cta"}
     for k, v in kw.items():
         setattr(p, names.get(k, k), int(v))
     return p

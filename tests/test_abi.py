@@ -80,3 +80,18 @@ def test_result_cache_parameter():
         with pytest.raises(YaspmvError) as e:
             Matrix.from_csr(2, 2, rp, c, v, device=-1, rc=rc)
         assert e.value.status == 1
+
+
+def test_tiles_per_cta_parameter():
+    """tiles_per_cta: 0 = auto, 1..64 explicit, anything else refused (host-only handles
+    report the requested value; device handles report the resolved one)."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix, YaspmvError
+    rp = np.array([0, 1, 2]); c = np.array([0, 1]); v = np.array([1.0, 2.0])
+    for k in (0, 1, 2, 64):
+        A = Matrix.from_csr(2, 2, rp, c, v, device=-1, tpc=k)
+        assert A.info()["params"]["tiles_per_cta"] == k
+        A.free()
+    for k in (-1, 65):
+        with pytest.raises(YaspmvError) as e:
+            Matrix.from_csr(2, 2, rp, c, v, device=-1, tpc=k)
+        assert e.value.status == 1

@@ -27,6 +27,8 @@ def main():
     ap.add_argument("--params", default=None)
     ap.add_argument("--md", default=None)
     ap.add_argument("--sweep", nargs="*", default=None, help="JSON param overrides, one re-encode each")
+    ap.add_argument("--ncu", action="store_true", help="launch every probe exactly twice, untimed (run under ncu; "
+                    "launch order = probe order)")
     args = ap.parse_args()
     import torch
 
@@ -73,10 +75,17 @@ def _probe(A, nnz, args):
 
     out = []
     probes = [("full", 0), ("no carries (7)", 7), ("7 - y stores (9)", 9),
-              ("up to the scan (8)", 8), ("stream+gather", 4),
+              ("up to the scan (8)", 8), ("8 + status store (10)", 10), ("8 + C stores (11)", 11),
+              ("stream+gather", 4),
               ("stream+L2-gather", 6), ("stream", 5), ("full (again)", 0)]
     for name, v in probes:
         if v == 6 and info["n"] < (1 << 20) * info["params"]["block_w"]:
+            continue
+        if args.ncu:
+            for _ in range(2):
+                run(v)
+            torch.cuda.synchronize()
+            print(json.dumps({"probe": name, "variant": v, "launches": 2}), flush=True)
             continue
         for _ in range(3):
             run(v)
