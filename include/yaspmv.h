@@ -194,7 +194,8 @@ yaspmv_status yaspmv_tune(yaspmv_matrix A, void* stream, yaspmv_params* chosen);
  * against). */
 yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode);
 
-/* yaspmv_reencode: re-encode A with new parameters (0 fields = keep current; see
+/* yaspmv_reencode: re-encode A with new parameters (0 fields — flags included — keep the
+ * current value; see
  * result_cache for its -1).  A change of result_cache / tiles_per_cta alone only
  * re-selects the launch (no re-encode). */
 yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params);

@@ -502,7 +502,7 @@ yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
   if (!want.C) want.C = cur.C;
   if (!want.col_mode) want.col_mode = cur.col_mode;
   if (!want.empty_mode) want.empty_mode = cur.empty_mode;
-  if (!params) want.flags = cur.flags;
+  if (!params || !want.flags) want.flags = cur.flags;
   want.rc = want.rc == 0 ? cur.rc : (want.rc < 0 ? 0 : want.rc);
   if (!want.tpc) want.tpc = cur.tpc;
   {  // only launch-time parameters change (strategy, tiles per CTA): no re-encode
