@@ -194,14 +194,41 @@ class FusedPowerIteration:
             if comm_factory is None:
                 from .matrix import Comm as comm_factory
             npdt = np.float32 if dtype == torch.float32 else np.float64
-            comm = comm_factory(self.device.index or 0, layout.rank, layout.world, layout.m_max, npdt, timeout_ms)
+            err = None
+            try:
+                comm = comm_factory(self.device.index or 0, layout.rank, layout.world, layout.m_max, npdt, timeout_ms)
+            except Exception as e:  # agreed on below, so that no rank is left waiting for a peer
+                comm, err = None, e
             if layout.world > 1:
                 import torch.distributed as dist
+                self._agree(err, group, "create the exchange buffers")
                 handles = [None] * layout.world
                 dist.all_gather_object(handles, comm.ipc_handle(), group=group)
-                comm.open_ipc(handles)
+                try:
+                    comm.open_ipc(handles)
+                except Exception as e:
+                    err = e
+                try:
+                    self._agree(err, group, "map the peers' buffers")
+                except RuntimeError:
+                    if hasattr(comm, "free"):
+                        comm.free()
+                    raise
+            elif err is not None:
+                raise err
         self.comm = comm
         self.restart()
+
+    @staticmethod
+    def _agree(err, group, what):
+        """Every rank learns whether every rank succeeded; all raise together (the caller
+        then falls back to the NCCL protocol on every rank, never on some)."""
+        import torch.distributed as dist
+        oks = [None] * dist.get_world_size(group)
+        dist.all_gather_object(oks, None if err is None else f"{type(err).__name__}: {err}", group=group)
+        bad = {r: m for r, m in enumerate(oks) if m is not None}
+        if bad:
+            raise RuntimeError(f"fused exchange: could not {what} on rank(s) {sorted(bad)}: {next(iter(bad.values()))}")
 
     def restart(self):
         """x_0 = 1/sqrt(N) on the real entries of this rank's copy, then (world > 1, own comm)

@@ -242,3 +242,51 @@ def test_fused_power_iteration_host_protocol_world2():
         x = y / np.linalg.norm(y)
     for xr in xs:
         assert np.allclose(xr, x, rtol=1e-12, atol=1e-15)
+
+
+class _FailingOpenComm(_ShmComm):
+    """Rank 1 cannot map its peers (e.g. no P2P between the GPUs)."""
+
+    def open_ipc(self, handles):
+        if self.rank == 1:
+            raise OSError("peer mapping refused")
+        super().open_ipc(handles)
+
+
+def _fused_fail_worker(rank, world, port, root, fail_create):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ["SHM_ROOT"] = root
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n = 1 << 10
+    from synth import matrices as sm
+    full = sm.circuit_like_rows(0, n, n=n, n_net=1, net_log2=(6, 7), band=64)
+    L = D.make_layout(full.row_ptr, rank, world)
+
+    def factory(*a):
+        if fail_create and rank == 0:
+            raise MemoryError("no device memory for the exchange buffers")
+        return _FailingOpenComm(*a)
+
+    try:
+        D.FusedPowerIteration(L, None, torch.float64, "cpu", comm_factory=factory)
+        outcome = "ok"
+    except RuntimeError as e:
+        outcome = str(e)
+    with open(os.path.join(root, f"r{rank}.txt"), "w") as f:
+        f.write(outcome)
+    dist.barrier()          # every rank got here: nobody is left waiting for a peer
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("fail_create", [False, True])
+def test_fused_setup_failure_is_agreed_by_every_rank(fail_create):
+    """If one rank cannot create or map the exchange buffers, every rank raises (so bench.py
+    falls back to the NCCL protocol everywhere) instead of the others blocking in a barrier."""
+    import torch.multiprocessing as mp
+    with tempfile.TemporaryDirectory() as td:
+        mp.spawn(_fused_fail_worker, args=(2, _free_port(), td, fail_create), nprocs=2, join=True)
+        outs = [open(os.path.join(td, f"r{r}.txt")).read() for r in range(2)]
+    want = "create the exchange buffers on rank(s) [0]" if fail_create else "map the peers' buffers on rank(s) [1]"
+    assert all(want in o for o in outs), outs
