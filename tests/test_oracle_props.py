@@ -174,3 +174,31 @@ def test_delta_escape_rule():
     assert d == [10, 32767, -1, -1]     # 32768 out of int16 range; -1 is the escape value
     assert np.array_equal(E.block_columns(e), e.col.astype(np.int64))
     del cols
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_inf_x_reaches_rows_through_stored_blocks_only(seed):
+    """DESIGN Q19, pinned by brute force: with one x_j = +Inf, the decoded 1x1 product is
+    non-finite exactly in the rows with a structural entry in column j (seg_row map, R2);
+    with FILLER blocks (R1, Q3: value 0, previous block's column) an empty row becomes NaN
+    iff its filler block carries column j.  tests/test_nonfinite_gpu.py compares the GPU
+    with this decode."""
+    a = synth.random_tiny(seed)
+    mask = a.to_dense() != 0
+    rows = np.repeat(np.arange(a.m), np.diff(a.row_ptr))
+    mask[rows, a.col] = True                       # structural zeros read x too
+    for j in range(a.n):
+        x = synth.make_x(a.n, np.float64, "int", seed)
+        x[j] = np.inf
+        reads = mask[:, j]
+        with np.errstate(invalid="ignore"):
+            e2 = E.encode(a.m, a.n, a.row_ptr, a.col, a.val, E.Params(1, 1, 1, 4, 2, 0, E.EMPTY_MAP))
+            assert np.array_equal(~np.isfinite(decode.spmv(e2, x)), reads)
+            e1 = E.encode(a.m, a.n, a.row_ptr, a.col, a.val, E.Params(1, 1, 1, 4, 2, 0, E.EMPTY_FILLER))
+            y1 = decode.spmv(e1, x)
+        stop_pos = np.flatnonzero(E.unpack_flags(e1) == 0)
+        empty = np.diff(a.row_ptr) == 0
+        filler_hits = np.zeros(a.m, dtype=bool)
+        filler_hits[empty] = E.block_columns(e1)[stop_pos[empty]] == j
+        assert np.array_equal(~np.isfinite(y1), reads | filler_hits)
+        assert np.all(np.isnan(y1[filler_hits]))
