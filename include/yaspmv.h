@@ -146,7 +146,10 @@ void yaspmv_free(yaspmv_matrix A);
  *   y: device, m elements; must not overlap x.
  * Deterministic: the same handle and x give a bitwise identical y.  One handle must not
  * run on two streams concurrently (it owns per-call scratch: ticket counter, carry
- * status words, BCCOO+ partial-result buffer).  Empty rows give y = 0.
+ * status words, BCCOO+ partial-result buffer).  Empty rows give y = 0 for every x (a FILLER
+ * block names block column NB, where x reads 0: DESIGN.md Q3); a row inside a stored h x w
+ * block reads the block's zero padding, 0 * x_j, so a non-finite x_j can reach
+ * it when h > 1.
  * Kernels: the fused SpMV (multiply, per-thread segmented sum, CTA segmented scan,
  * decoupled look-back carries, write-back; §3) and, when S > 1, the slice
  * combine. */

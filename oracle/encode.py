@@ -11,10 +11,11 @@ where the paper is silent or garbled are SURVEY §8(c) Q1-Q16 and are listed in 
   E4  h value arrays, w values per block, zeros inside a block stored
   E5  col = ORIGINAL block column, also for BCCOO+ 
   E6  bit flag 0 = row stop (last block of its stacked row), 1 = continue
-      empty stacked rows: R1 a zero filler block (paper's "multiple 1s")
+      empty stacked rows: R1 a zero filler block (paper's "multiple 1s") whose
+                          column is NB, past the last block column (Q3)
                           R2 a seg_row map + zero list                    (Q1)
   E7  pad with '1' bits to a multiple of the workgroup tile T*C; pad blocks
-      hold zero values and repeat the previous column (Q3)
+      hold zero values and repeat the last column of the stream (Q3)
   E8  flags packed LSB-first in bytes (Q2)
   E9  col storage: unsigned short if NB < 65535 (Q6) else int32; or the
       segmented int16 difference with -1 escape (Q7)
@@ -172,10 +173,9 @@ def encode(m: int, n: int, row_ptr, col, val, p: Params) -> Encoded:
         stream_sr = all_sr[order]
         stream_fill = is_fill[order]
         stream_bc = np.concatenate([blk_bc, np.zeros(empty.size, np.int64)])[order]
-        # filler column = column of the preceding block in the stream (0 if first) (Q3)
-        idx = np.where(~stream_fill, np.arange(order.size), -1)
-        np.maximum.accumulate(idx, out=idx)
-        stream_bc = np.where(stream_fill, np.where(idx >= 0, stream_bc[np.maximum(idx, 0)], 0), stream_bc)
+        # filler column = NB, one past the last block column: x reads 0 there (Q4), so an
+        # empty row is exactly 0 for every x, also x = +-Inf (Q3, round 2)
+        stream_bc = np.where(stream_fill, NB, stream_bc)
         n_filler = int(empty.size)
     else:
         pos_of_real = np.arange(n_real, dtype=np.int64)

@@ -342,13 +342,11 @@ yaspmv_status encode(const CSR& A, const Params& p, Canonical& out) {
         }
       }
     }
-    // R1 fillers repeat the previous block's column; pad blocks repeat the last (Q3)
+    // R1 fillers take block column NB, past the last one: x reads 0 there (Q4), so an
+    // empty row is 0 for every x, +-Inf included; pad blocks repeat the last column (Q3)
     if (filler && n_empty) {
       for (int64_t sr = 0; sr < nsr; ++sr)
-        if (cnt[sr] == 0) {
-          const int64_t b = off[sr];
-          colb[b] = b > 0 ? colb[b - 1] : 0;
-        }
+        if (cnt[sr] == 0) colb[off[sr]] = (int32_t)out.NB;
     }
     for (int64_t b = out.nnzb; b < NP; ++b) colb[b] = out.nnzb > 0 ? colb[out.nnzb - 1] : 0;
 

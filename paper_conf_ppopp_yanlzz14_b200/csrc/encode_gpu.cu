@@ -114,9 +114,9 @@ __global__ void k_fill_blocks(const unsigned long long* bkey, int64_t nreal, int
 __global__ void k_fillers(const int32_t* cnt, int64_t nsr, const int64_t* off_real, const int64_t* off_full,
                           const unsigned long long* bkey, int64_t NB, int32_t* colb, uint8_t* flags) {
   for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < nsr; s += (int64_t)gridDim.x * blockDim.x)
-    if (cnt[s] == 0) {  // Q1 R1 / Q3: zero block repeating the previous real block's column
+    if (cnt[s] == 0) {  // Q1 R1 / Q3: zero block in block column NB (x reads 0 there, Q4)
       const int64_t pos = off_full[s];
-      colb[pos] = off_real[s] > 0 ? (int32_t)(bkey[off_real[s] - 1] % NB) : 0;
+      colb[pos] = (int32_t)NB;
       clear_bit(flags, pos);
     }
 }

@@ -142,7 +142,8 @@ __device__ __forceinline__ VT word_val(const uint32_t* w, int i) {
 template <typename VT, int W>
 __device__ __forceinline__ void gather_x(const VT* x, int64_t cb, int64_t n, uint64_t pol, VT (&xs)[W]) {
   if constexpr (W == 1) {
-    xs[0] = ldx(x + cb, pol);
+    // predicated: a FILLER block sits in block column NB (Q3) and reads 0, never x
+    xs[0] = cb < n ? ldx(x + cb, pol) : VT(0);
   } else {
     const int64_t i0 = cb * W;
     if (i0 + W <= n) {

@@ -87,3 +87,20 @@ def test_coo_normalisation_matches_oracle():
     rpo, colo, valo = E.normalize(m, n, rows[srt], cols[srt], vals[srt])
     enc2 = E.encode(m, n, rpo, colo, valo, E.Params(2, 2, 2, 4, 64, E.COL_I32, 0))
     assert np.array_equal(B.export("val0"), enc2.val[0])
+
+
+
+def test_delta_reset_per_thread_tile_cpp_encoder():
+    """The C++ encoder resets the P:121 difference at every thread tile of T blocks (the
+    rule pinned by tests/golden/p121_delta_reset.txt on the oracle): 512 rows of one block
+    each, col = 100 + b, T = 4, C = 64 -> stored 100 + b at b % 4 == 0, else 1."""
+    m = 512
+    rp = np.arange(m + 1, dtype=np.int64)
+    col = (100 + np.arange(m)).astype(np.int32)
+    A = Matrix.from_csr(m, 1000, rp, col, np.ones(m, np.float32), device=-1, T=4, C=64,
+                        col_mode=E.COL_DELTA, empty_mode=E.EMPTY_FILLER)
+    try:
+        want = np.where(np.arange(m) % 4 == 0, col, 1)
+        assert np.array_equal(A.export("col_delta").astype(np.int64), want)
+    finally:
+        A.free()

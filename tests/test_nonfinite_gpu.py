@@ -11,12 +11,12 @@ These tests poison a few rows and check that (a) the poisoned rows come out NaN 
 the clean matrix.
 
 x = +Inf: every stored block multiplies x, including the zero padding of an h x w block
- and the FILLER block of an empty stacked row (Q1/Q3 in DESIGN.md: value 0,
-column of the previous real block), so 0 * Inf = NaN can reach a row that reads no Inf
-column through a structural entry.  The expected NaN / +Inf pattern is therefore the one
+(P:83-105), so 0 * Inf = NaN can reach a row of a stored h x w block that has no
+structural entry in the Inf column.  The expected NaN / +Inf pattern is therefore the one
 the oracle's decode of the canonical arrays (oracle/decode.py, IEEE arithmetic over every
-stored block) produces; with the seg_row map (no fillers) and 1x1 blocks it is exactly the
-CSR pattern.
+stored block) produces.  A FILLER block of an empty stacked row sits in block column NB,
+where x reads 0 (Q3/Q19), so with 1x1 blocks the pattern is exactly the CSR one
+(y = A.x, O1) for both empty-row encodings, and every row of an empty block row is 0.
 """
 import numpy as np
 import pytest
@@ -113,8 +113,14 @@ def test_inf_x_reaches_exactly_the_rows_that_read_it(web, pi):
     assert np.array_equal(np.isposinf(y), np.isposinf(y_dec))
     assert not np.any(np.isneginf(y))
     assert np.all(~np.isfinite(y[reads]))
-    if enc.p.h == enc.p.w == 1 and enc.p.empty_mode == E.EMPTY_MAP:
+    if enc.p.h == enc.p.w == 1:              # exactly O1's pattern, FILLER or MAP
         assert np.array_equal(np.flatnonzero(~np.isfinite(y)), reads)
+    # "empty rows give y = 0" (include/yaspmv.h): every row of an empty block row, any x
+    h = enc.p.h
+    blk_nnz = np.add.reduceat(np.diff(csr.row_ptr), np.arange(0, csr.m, h)) if csr.m else np.zeros(0)
+    empty_rows = np.flatnonzero(np.repeat(blk_nnz == 0, h)[: csr.m])
+    assert empty_rows.size > 0
+    assert np.all(y[empty_rows] == 0)
     x_clean = x.copy()
     x_clean[cols] = 0
     _check_clean_rows(csr, y, x_clean, np.flatnonzero(~np.isfinite(y_dec)))

@@ -168,3 +168,18 @@ def test_strategy2_equals_strategy1_across_workgroups(T, C, RC):
     pad = (-len(vals)) % (T * C)
     s2, _ = simulate.simulate_s2(vals + [0] * pad, bits + [1] * pad, T, C, RC)
     assert s2 == g7["segment_sums"]
+
+
+def test_delta_reset_per_thread_tile_p121():
+    """P:121 segmented difference resets at every THREAD tile (T blocks), not every
+    workgroup tile (T*C) and not every block: hand-derived fixture with T = 2, C = 2 over
+    two workgroup tiles (tests/golden/p121_delta_reset.txt)."""
+    g = load_golden("p121_delta_reset.txt")
+    m = g["rows"]
+    rp = np.arange(m + 1, dtype=np.int64)
+    col = np.array(g["col"], dtype=np.int32)
+    e = E.encode(m, g["ncols"], rp, col, np.ones(m), E.Params(1, 1, 1, g["T"], g["C_threads"], E.COL_DELTA, 1))
+    assert e.ntiles == 2 and e.nnzb_pad == m
+    assert e.col_delta.tolist() == g["delta"]
+    assert e.col.tolist() == g["col"]                    # int32 array kept for escapes (Q7)
+    assert E.block_columns(e).tolist() == g["col"]

@@ -179,10 +179,9 @@ def test_delta_escape_rule():
 @pytest.mark.parametrize("seed", range(20))
 def test_inf_x_reaches_rows_through_stored_blocks_only(seed):
     """DESIGN Q19, pinned by brute force: with one x_j = +Inf, the decoded 1x1 product is
-    non-finite exactly in the rows with a structural entry in column j (seg_row map, R2);
-    with FILLER blocks (R1, Q3: value 0, previous block's column) an empty row becomes NaN
-    iff its filler block carries column j.  tests/test_nonfinite_gpu.py compares the GPU
-    with this decode."""
+    non-finite exactly in the rows with a structural entry in column j — with the seg_row
+    map (R2) and with FILLER blocks (R1), whose column NB reads x as 0 (Q3) — and every
+    empty row is exactly 0.  tests/test_nonfinite_gpu.py compares the GPU with this decode."""
     a = synth.random_tiny(seed)
     mask = a.to_dense() != 0
     rows = np.repeat(np.arange(a.m), np.diff(a.row_ptr))
@@ -198,7 +197,7 @@ def test_inf_x_reaches_rows_through_stored_blocks_only(seed):
             y1 = decode.spmv(e1, x)
         stop_pos = np.flatnonzero(E.unpack_flags(e1) == 0)
         empty = np.diff(a.row_ptr) == 0
-        filler_hits = np.zeros(a.m, dtype=bool)
-        filler_hits[empty] = E.block_columns(e1)[stop_pos[empty]] == j
-        assert np.array_equal(~np.isfinite(y1), reads | filler_hits)
-        assert np.all(np.isnan(y1[filler_hits]))
+        if e1.n_filler:
+            assert np.all(E.block_columns(e1)[stop_pos[empty]] == e1.NB)   # Q3: column NB
+        assert np.array_equal(~np.isfinite(y1), reads)
+        assert np.all(y1[empty] == 0)
