@@ -1,0 +1,121 @@
+"""Pins of the panel-sliced BCCOO+ oracle (oracle/panel.py, DESIGN.md §2.1 readings P1-P6):
+a hand-derived example on the paper's matrix A (tests/golden/panel_eq1_A.txt), the
+degenerate case that must reproduce the paper's plain BCCOO arrays bit for bit (one panel,
+one slice: P:83-119 through oracle/encode.py), brute force y = A x with exact integer
+arithmetic, and the format's invariants.  CPU only."""
+import numpy as np
+import pytest
+
+import synth
+from golden_io import load_golden
+from oracle import decode, encode as E, panel as PN
+
+
+def _csr_of(A):
+    m, n = A.shape
+    r, c = np.nonzero(A)
+    rp = np.zeros(m + 1, dtype=np.int64)
+    np.cumsum(np.bincount(r, minlength=m), out=rp[1:])
+    return m, n, rp, c.astype(np.int32), A[r, c]
+
+
+def _bits(enc):
+    return np.unpackbits(enc.flags, bitorder="little")[: enc.nband_pad]
+
+
+def test_hand_example_eq1_A():
+    g = load_golden("panel_eq1_A.txt")
+    A = np.array(load_golden("eq1_A.txt")["A"], dtype=np.float64).reshape(4, 8)
+    pp = PN.PanelParams(R=g["R"], W=g["W"], B=g["B"], T=g["T"], C=g["C_threads"],
+                        far=E.Params(1, 1, 1, 4, 64, E.COL_I32, E.EMPTY_FILLER))
+    enc = PN.encode_panel(*_csr_of(A), pp)
+    assert enc.KS == g["KS"]
+    assert _bits(enc).tolist() == g["flags"]
+    assert enc.col16.tolist() == g["col16"]
+    assert enc.val.tolist() == g["val"]
+    assert enc.panel_blk0.tolist() == g["panel_blk0"]
+    assert enc.slice_ptr.ravel().tolist() == g["slice_ptr"]
+    assert enc.stop_ptr.ravel().tolist() == g["stop_ptr"]
+    assert enc.occ.ravel().tolist() == g["occ"]
+    assert enc.far_csr[2].tolist() == g["far_val"]
+    x = np.arange(1, 9, dtype=np.float64)
+    assert decode.spmv(enc.far, x).tolist() == g["y_far"]
+    assert PN.spmv(enc, x).tolist() == g["y"]
+    assert np.array_equal(PN.to_dense(enc), A)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_one_panel_one_slice_is_plain_bccoo(seed):
+    """R >= m, B = 0, W >= R: every entry is a band entry of the single slice, and the
+    band arrays are exactly the paper's BCCOO arrays (1x1 blocks, S = 1) with the seg_row
+    reading (Q1/R2): same flags, columns (u16), values;
+    the occupancy bitmap marks exactly the rows of seg_row."""
+    a = synth.random_tiny(seed)
+    R = 32 * (-(-a.m // 32))
+    pp = PN.PanelParams(R=R, W=max(R, 4 * (-(-a.n // 4))), B=0, T=4, C=2)
+    enc = PN.encode_panel(a.m, a.n, a.row_ptr, a.col, a.val, pp)
+    plain = E.encode(a.m, a.n, a.row_ptr, a.col, a.val, E.Params(1, 1, 1, 4, 2, E.COL_U16, E.EMPTY_MAP))
+    assert enc.KS == 1 and enc.far.nnzb == 0 and enc.nband == a.nnz
+    assert enc.nband_pad == plain.nnzb_pad
+    assert np.array_equal(enc.flags, plain.flags)
+    assert np.array_equal(enc.col16, plain.col)
+    assert np.array_equal(enc.val, plain.val[0])
+    rows_with = np.flatnonzero(np.diff(a.row_ptr) > 0)
+    occ = np.unpackbits(enc.occ[0, 0].view(np.uint8), bitorder="little")[: a.m]
+    assert np.array_equal(np.flatnonzero(occ), rows_with)
+    if plain.seg_row.size:
+        assert np.array_equal(plain.seg_row, rows_with)
+
+
+def _banded(seed, m, n, band, extra=0.1):
+    g = np.random.default_rng(seed)
+    A = np.zeros((m, n))
+    for i in range(m):
+        k = g.integers(0, 6)
+        cols = np.clip(i + g.integers(-band, band + 1, size=k), 0, n - 1)
+        A[i, cols] = g.integers(-3, 4, size=k)
+        if g.random() < extra:
+            A[i, g.integers(0, n)] = g.integers(1, 4)
+    A[g.integers(0, m, size=max(1, m // 7))] = 0          # empty rows
+    return A
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_brute_force_integer_exact(seed):
+    g = np.random.default_rng(100 + seed)
+    m, n = int(g.integers(1, 90)), int(g.integers(1, 90))
+    A = _banded(seed, m, n, int(g.integers(0, 12)))
+    pp = PN.PanelParams(R=int(g.integers(1, 20)), W=int(g.integers(1, 9)), B=int(g.integers(0, 10)),
+                        T=int(g.choice([1, 2, 4])), C=int(g.choice([1, 2, 3])),
+                        diag0=int(g.integers(-3, 4)),
+                        far=E.Params(1, 1, 1, 4, 2, 0, int(g.choice([E.EMPTY_FILLER, E.EMPTY_MAP]))))
+    enc = PN.encode_panel(*_csr_of(A), pp)
+    x = g.integers(-4, 5, size=n).astype(np.float64)
+    assert np.array_equal(PN.spmv(enc, x), A @ x)
+    assert np.array_equal(PN.to_dense(enc), A)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_invariants(seed):
+    a = synth.circuit_like_rows(0, 3000, kind="integer", n=3000, band=300, n_net=2, net_log2=(9, 10))
+    pp = PN.PanelParams(R=256, W=64, B=300, T=4, C=8, far=E.Params(1, 1, 1, 4, 8, 0, 0))
+    if seed % 2:
+        pp.diag0 = 17
+    enc = PN.encode_panel(a.m, a.n, a.row_ptr, a.col, a.val, pp)
+    bits = _bits(enc)
+    rows, p, k, band = PN.split(a.m, a.n, a.row_ptr, a.col, a.val, pp)
+    # every entry once: band + far = nnz; far entries lie outside their panel's band
+    assert enc.nband == int(band.sum()) and enc.far_csr[1].size == a.nnz - enc.nband
+    # stops = set bits of the occupancy bitmaps, slice by slice
+    for q in range(enc.npanels):
+        b0 = enc.panel_blk0[q]
+        assert (enc.panel_blk0[q + 1] - b0) % (pp.T * pp.C) == 0
+        for kk in range(enc.KS):
+            seg = bits[b0 + enc.slice_ptr[q, kk]: b0 + enc.slice_ptr[q, kk + 1]]
+            pops = sum(bin(int(w)).count("1") for w in enc.occ[q, kk])
+            assert int((seg == 0).sum()) == pops == enc.stop_ptr[q, kk + 1] - enc.stop_ptr[q, kk]
+        assert np.all(bits[b0 + enc.slice_ptr[q, -1]: enc.panel_blk0[q + 1]] == 1)   # pad bits
+    assert np.all(enc.col16.astype(np.int64) < pp.W)
+    x = synth.make_x(a.n, np.float64, "int", seed)
+    A = a.to_dense()
+    assert np.array_equal(PN.spmv(enc, x), A @ x)
