@@ -87,6 +87,16 @@ typedef struct {
                            a tile issues the next tile's loads at once while the tile's
                            stores drain.  Results are bitwise identical for every k.
                            Launch-time (no re-encode); forced to 1 with YASPMV_TICKET_IDS. */
+  /* Panel-sliced BCCOO+ (BCCOO+'s vertical slices, stacked
+     inside each panel of R rows, slices of W columns placed relative to the panel): the
+     entries of panel p with a column in [p*R + band_col0 - band, ... + KS*W), KS =
+     ceil((R + 2*band)/W), go to the band stream, whose every gather is served from a
+     W-value window of x in shared memory; the rest is a plain BCCOO/BCCOO+ matrix encoded
+     with the fields above.  fp32, 1x1 blocks; not with the fused multi-GPU step. */
+  int32_t band;        /* band half-width B in columns; 0 = off (plain format)           */
+  int32_t panel_rows;  /* R: multiple of 256, <= 32768; 0 = 16384                        */
+  int32_t slice_width; /* W: multiple of 4, <= 65536, KS <= 64; 0 = 8192                 */
+  int32_t band_col0;   /* column of row 0 (a row-partitioned rank: its first global row) */
 } yaspmv_params;
 
 typedef struct {
@@ -110,6 +120,12 @@ typedef struct {
   double tune_seconds;       /* wall time of the last yaspmv_tune                         */
   int32_t tune_candidates;   /* candidates timed by the last yaspmv_tune                   */
   int32_t reserved;
+  /* panel-sliced BCCOO+ (params.band > 0): the fields above describe the far part        */
+  int64_t band_blocks;       /* band entries (1x1 blocks)                                 */
+  int64_t band_blocks_pad;   /* after padding every panel to the band tile                */
+  int64_t band_panels;       /* panels = CTAs of the band kernel                          */
+  int64_t band_slices;       /* KS, slices per panel                                      */
+  int64_t band_stops;        /* row stops of the band stream                              */
 } yaspmv_info;
 
 /* ---------------------------------------------------------------- build / free
@@ -219,7 +235,19 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* out);
 enum {
   YASPMV_ARR_FLAGS = 0, YASPMV_ARR_COL = 1, YASPMV_ARR_COL_DELTA = 2,
   YASPMV_ARR_VAL0 = 3, YASPMV_ARR_VAL1 = 4, YASPMV_ARR_VAL2 = 5, YASPMV_ARR_VAL3 = 6,
-  YASPMV_ARR_SEG_ROW = 7, YASPMV_ARR_ZERO_ROWS = 8, YASPMV_ARR_CTA_SEG0 = 9, YASPMV_ARR_FRE = 10
+  YASPMV_ARR_SEG_ROW = 7, YASPMV_ARR_ZERO_ROWS = 8, YASPMV_ARR_CTA_SEG0 = 9, YASPMV_ARR_FRE = 10,
+  /* panel-sliced BCCOO+ band stream (params.band > 0; readings P1-P6 of DESIGN.md §2.1):
+   *  BAND_FLAGS      uint8 [band_blocks_pad/8]  0 = last entry of its row in its slice
+   *  BAND_COL16      uint16 [band_blocks_pad]   column - (p*R + col0 - B) - k*W
+   *  BAND_VAL        value [band_blocks_pad]
+   *  BAND_PANEL_BLK0 int64 [panels + 1]         first block of each panel (padded)
+   *  BAND_SLICE_PTR  int32 [panels * (KS+1)]    block offset of slice k inside its panel
+   *  BAND_STOP_PTR   int32 [panels * (KS+1)]    row stops before slice k inside its panel
+   *  BAND_OCC        uint32 [panels * KS * R/32] row-occupancy bitmap of every slice
+   *  BAND_PRE        uint16 [panels * KS * R/32] set bits before each bitmap word */
+  YASPMV_ARR_BAND_FLAGS = 11, YASPMV_ARR_BAND_COL16 = 12, YASPMV_ARR_BAND_VAL = 13,
+  YASPMV_ARR_BAND_PANEL_BLK0 = 14, YASPMV_ARR_BAND_SLICE_PTR = 15, YASPMV_ARR_BAND_STOP_PTR = 16,
+  YASPMV_ARR_BAND_OCC = 17, YASPMV_ARR_BAND_PRE = 18
 };
 
 /* yaspmv_export: copy canonical array `which` into host_dst (capacity `bytes`).  Returns
@@ -310,6 +338,12 @@ const char* yaspmv_last_error(void);
 const char* yaspmv_version(void);
 /* Kernel launches issued by the last yaspmv_spmv on this handle (1, or 2 with S > 1). */
 int32_t yaspmv_launches_per_spmv(yaspmv_matrix A);
+/* Debug spin bound: with the environment variable YASPMV_SPIN_LIMIT=N (> 0, read
+ * once per process) a carry look-back that polls its predecessors' status words
+ * more than N times traps the kernel instead of hanging (the stream reports
+ * cudaErrorLaunchFailure, sticky for the process) after writing the waiting tile id to
+ * mapped host memory.  Returns that tile id, or -1 if no bound was hit (or none is set). */
+int64_t yaspmv_debug_spin_tile(void);
 
 #ifdef __cplusplus
 }

@@ -36,7 +36,10 @@ extern "C" {
  *             (no carry publish, no y stores, no look-back);
  *   variant 9 roofline probe: variant 7 without the y stores of the write-back;
  *   variant 10 roofline probe: variant 8 + thread C-1's 16-byte status store (publish);
- *   variant 11 roofline probe: variant 8 + one coalesced 4-byte store per thread.
+ *   variant 11 roofline probe: variant 8 + one coalesced 4-byte store per thread;
+ *   variant 12 test of the debug spin bound: variant 3 whose tile 0 never publishes its
+ *             carry-out, so the look-back of a later tile of a row spanning >= 3 tiles
+ *             polls forever (traps under YASPMV_SPIN_LIMIT, yaspmv.h).
  * Variants 4 and 5 do not compute y; they exist to measure.
  * x, y: device; the column storage is whatever A was built with (the caller builds A with
  * col_mode I32 for steps 1-2 and the auto/short mode for step 3). */

@@ -19,7 +19,11 @@ COL_AUTO, COL_U16, COL_I32, COL_DELTA16 = 0, 1, 2, 3
 EMPTY_AUTO, EMPTY_FILLER, EMPTY_MAP = 0, 1, 2
 KEEP_HOST, DROP_CSR, GPU_ENCODE, TICKET_IDS, NO_PDL, FORCE_HANDOFF = 1, 2, 4, 8, 16, 32
 ARR = {"flags": 0, "col": 1, "col_delta": 2, "val0": 3, "val1": 4, "val2": 5, "val3": 6,
-       "seg_row": 7, "zero_rows": 8, "cta_seg0": 9, "fre": 10}
+       "seg_row": 7, "zero_rows": 8, "cta_seg0": 9, "fre": 10,
+       # panel-sliced BCCOO+ band stream
+       "band_flags": 11, "band_col16": 12, "band_val": 13, "band_panel_blk0": 14, "band_slice_ptr": 15,
+       "band_stop_ptr": 16, "band_occ": 17, "band_pre": 18}
+PANEL_BT, PANEL_BC = 16, 512  # band stream tile of the panel kernel (csrc/panel.hpp)
 
 MAX_RANKS = 8  # YASPMV_MAX_RANKS
 IPC_HANDLE_BYTES = 64
@@ -33,7 +37,7 @@ EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv"
             "yaspmv_comm_create", "yaspmv_comm_ipc_handle", "yaspmv_comm_open_ipc", "yaspmv_comm_connect_local",
             "yaspmv_comm_x", "yaspmv_comm_begin", "yaspmv_power_step_fused", "yaspmv_comm_wait",
             "yaspmv_comm_norm2_device", "yaspmv_comm_seq", "yaspmv_comm_check", "yaspmv_launches_per_fused_step",
-            "yaspmv_comm_free",
+            "yaspmv_comm_free", "yaspmv_debug_spin_tile",
             # include/yaspmv_ablation.h
             "yaspmv_ablation_spmv", "yaspmv_ablation_tree", "yaspmv_ablation_tree_scratch_bytes"]
 
@@ -42,7 +46,8 @@ class Params(ctypes.Structure):
     _fields_ = [("block_h", ctypes.c_int32), ("block_w", ctypes.c_int32), ("slices", ctypes.c_int32),
                 ("thread_tile", ctypes.c_int32), ("cta_size", ctypes.c_int32), ("col_mode", ctypes.c_int32),
                 ("empty_mode", ctypes.c_int32), ("flags", ctypes.c_int32), ("result_cache", ctypes.c_int32),
-                ("tiles_per_cta", ctypes.c_int32)]
+                ("tiles_per_cta", ctypes.c_int32), ("band", ctypes.c_int32), ("panel_rows", ctypes.c_int32),
+                ("slice_width", ctypes.c_int32), ("band_col0", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
@@ -57,7 +62,9 @@ class Info(ctypes.Structure):
                 ("footprint_bytes", ctypes.c_int64), ("params", Params), ("dtype", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("has_seg_row", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
                 ("build_seconds", ctypes.c_double), ("tune_seconds", ctypes.c_double),
-                ("tune_candidates", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("tune_candidates", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("band_blocks", ctypes.c_int64), ("band_blocks_pad", ctypes.c_int64), ("band_panels", ctypes.c_int64),
+                ("band_slices", ctypes.c_int64), ("band_stops", ctypes.c_int64)]
 
     def as_dict(self):
         d = {}
@@ -120,6 +127,7 @@ def _load():
         "yaspmv_comm_check": ([H], ctypes.c_int),
         "yaspmv_launches_per_fused_step": ([H], i32),
         "yaspmv_comm_free": ([H], None),
+        "yaspmv_debug_spin_tile": ([], i64),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

@@ -28,7 +28,47 @@ yaspmv_status fail(yaspmv_status st, const std::string& msg) {
   g_err = msg;
   return st;
 }
+// Debug spin bound: YASPMV_SPIN_LIMIT=N (read once per process) makes a
+// look-back that polls more than N times write its tile id to a mapped host slot and trap;
+// the slot survives the sticky launch error and is read by yaspmv_debug_spin_tile().
+long long debug_spin_limit() {
+  static const long long lim = [] {
+    const char* e = std::getenv("YASPMV_SPIN_LIMIT");
+    return e ? std::atoll(e) : 0ll;
+  }();
+  return lim;
+}
+static long long* g_spin_slot = nullptr;
+long long* debug_spin_slot() {
+  if (debug_spin_limit() <= 0) return nullptr;
+  static const bool ok = [] {
+    void* p = nullptr;
+    if (cudaHostAlloc(&p, sizeof(long long), cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) return false;
+    g_spin_slot = static_cast<long long*>(p);
+    *g_spin_slot = -1;
+    return true;
+  }();
+  return ok ? g_spin_slot : nullptr;
+}
 }  // namespace yaspmv
+
+extern "C" int64_t yaspmv_debug_spin_tile(void) {
+  return yaspmv::g_spin_slot ? (int64_t) * (volatile long long*)yaspmv::g_spin_slot : -1;
+}
+
+namespace {
+// run a call on the handle's device and restore the caller's current device afterwards
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (dev >= 0 && cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+}  // namespace
 
 #define CUDA_TRY(expr)                                                                       \
   do {                                                                                       \
@@ -57,6 +97,10 @@ Params from_abi(const yaspmv_params* p) {
     q.flags = p->flags;
     q.rc = p->result_cache;
     q.tpc = p->tiles_per_cta;
+    q.band = p->band;
+    q.pR = p->panel_rows;
+    q.pW = p->slice_width;
+    q.col0 = p->band_col0;
   }
   return q;
 }
@@ -73,6 +117,10 @@ yaspmv_params to_abi(const Params& q) {
   p.flags = q.flags;
   p.result_cache = q.rc;
   p.tiles_per_cta = q.tpc;
+  p.band = q.band;
+  p.panel_rows = q.pR;
+  p.slice_width = q.pW;
+  p.band_col0 = q.col0;
   return p;
 }
 
@@ -221,12 +269,120 @@ yaspmv_status install_canonical_impl(yaspmv_matrix A, Canonical&& c, int flags) 
   return YASPMV_OK;
 }
 
+// panel-sliced BCCOO+: validate and resolve the band parameters (0 = default)
+yaspmv_status resolve_band(yaspmv_matrix A, Params& p) {
+  if (p.band < 0) return fail(YASPMV_EINVAL, "band must be >= 0");
+  if (p.band == 0) {
+    p.pR = p.pW = p.col0 = 0;
+    return YASPMV_OK;
+  }
+  if (A->dtype != YASPMV_F32) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ is compiled for fp32");
+  if (p.h != 1 || p.w != 1) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ needs 1x1 blocks");
+  if (p.pR == 0) p.pR = 16384;
+  if (p.pW == 0) p.pW = 8192;
+  if (p.pR % 256 || p.pR <= 0 || p.pR > 32768) return fail(YASPMV_EINVAL, "panel_rows must be a multiple of 256 in [256, 32768]");
+  if (p.pW % 4 || p.pW <= 0 || p.pW > 65536) return fail(YASPMV_EINVAL, "slice_width must be a multiple of 4 in [4, 65536]");
+  if ((p.pR + 2LL * p.band + p.pW - 1) / p.pW > PANEL_MAX_KS)
+    return fail(YASPMV_EINVAL, "panel-sliced BCCOO+: (panel_rows + 2*band) / slice_width exceeds 64 slices");
+  if (A->device >= 0) {
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, A->device);
+    if (panel_smem_bytes(p.pR, p.pW) + 2048 > (size_t)optin)
+      return fail(YASPMV_EINVAL, "panel_rows / slice_width need more shared memory than a CTA has");
+  }
+  return YASPMV_OK;
+}
+
+// upload the band part into nd (the caller installs it)
+yaspmv_status panel_to_device(yaspmv_matrix A, const PanelCanonical& pc, PanelDev& nd) {
+  nd = PanelDev();
+  auto up = [&](const void* src, size_t bytes, void** dst) -> yaspmv_status {
+    *dst = nullptr;
+    if (!bytes) return YASPMV_OK;
+    CUDA_TRY(cudaMalloc(dst, bytes));
+    CUDA_TRY(cudaMemcpy(*dst, src, bytes, cudaMemcpyHostToDevice));
+    return YASPMV_OK;
+  };
+  const int64_t ntl = pc.nband_pad / PANEL_TC;
+  yaspmv_status st;
+  if ((st = upload_permuted(reinterpret_cast<const uint8_t*>(pc.col16.data()), ntl, PANEL_BC, 2 * PANEL_BT,
+                            &nd.col16)) != YASPMV_OK ||
+      (st = upload_permuted(pc.val.data(), ntl, PANEL_BC, PANEL_BT * A->vsize, &nd.val)) != YASPMV_OK ||
+      (st = up(pc.flags.data(), pc.flags.size(), (void**)&nd.flags)) != YASPMV_OK ||
+      (st = up(pc.panel_blk0.data(), pc.panel_blk0.size() * 8, (void**)&nd.panel_blk0)) != YASPMV_OK ||
+      (st = up(pc.slice_ptr.data(), pc.slice_ptr.size() * 4, (void**)&nd.slice_ptr)) != YASPMV_OK ||
+      (st = up(pc.stop_ptr.data(), pc.stop_ptr.size() * 4, (void**)&nd.stop_ptr)) != YASPMV_OK ||
+      (st = up(pc.occ.data(), pc.occ.size() * 4, (void**)&nd.occ)) != YASPMV_OK ||
+      (st = up(pc.pre.data(), pc.pre.size() * 2, (void**)&nd.pre)) != YASPMV_OK) {
+    nd.free_all();
+    return st;
+  }
+  const int64_t np = std::max<int64_t>(pc.g.npanels, 1);
+  if (cudaMalloc((void**)&nd.part, np * sizeof(double)) != cudaSuccess ||
+      cudaMalloc((void**)&nd.scratch, nrm2sq_blocks(np) * sizeof(double)) != cudaSuccess) {
+    nd.free_all();
+    return fail(YASPMV_ENOMEM, "panel scratch allocation failed");
+  }
+  int e = panel_attr(pc.g.R, pc.g.W, &A->pan_regs);
+  if (e != 0) {
+    nd.free_all();
+    return fail(YASPMV_ECUDA, std::string("panel kernel attributes: ") + cudaGetErrorString((cudaError_t)e));
+  }
+  CUDA_TRY(cudaDeviceSynchronize());
+  return YASPMV_OK;
+}
+
+yaspmv_status encode_plain_into(yaspmv_matrix A, const CSR& src, const Params& p, double t0);
+
 // (re-)encode A->csr with params and upload; on failure A is left unchanged
 yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
   const double t0 = now_s();
   Params p;
   yaspmv_status st = resolve_params(want, A->csr.m, A->csr.n, p);
   if (st != YASPMV_OK) return st;
+  if ((st = resolve_band(A, p)) != YASPMV_OK) return st;
+  A->nnz_total = A->csr.nnz;
+  if (p.band == 0) {
+    if ((st = encode_plain_into(A, A->csr, p, t0)) != YASPMV_OK) return st;
+    A->band_on = false;
+    A->pan = PanelCanonical();
+    A->have_pan_host = false;
+    if (A->device >= 0) A->pd.free_all();
+    return YASPMV_OK;
+  }
+  // panel-sliced BCCOO+: split into the far part (plain path) and the band stream
+  PanelGeom g;
+  g.R = p.pR;
+  g.W = p.pW;
+  g.B = p.band;
+  g.col0 = p.col0;
+  CSR far;
+  PanelCanonical pc;
+  if ((st = encode_panel(A->csr, g, far, pc)) != YASPMV_OK) return st;
+  PanelDev nd;
+  if (A->device >= 0) {
+    CUDA_TRY(cudaSetDevice(A->device));
+    if ((st = panel_to_device(A, pc, nd)) != YASPMV_OK) return st;
+  }
+  if ((st = encode_plain_into(A, far, p, t0)) != YASPMV_OK) {
+    nd.free_all();
+    return st;
+  }
+  if (A->device >= 0) {
+    A->pd.free_all();
+    A->pd = nd;
+  }
+  A->band_on = true;
+  A->have_pan_host = A->device < 0 || (p.flags & YASPMV_KEEP_HOST);
+  if (!A->have_pan_host) pc.release_arrays();
+  A->pan = std::move(pc);
+  A->build_s = now_s() - t0;
+  return YASPMV_OK;
+}
+
+// the plain BCCOO/BCCOO+ encoding of `src` (A->csr, or the far part of a panel encoding)
+yaspmv_status encode_plain_into(yaspmv_matrix A, const CSR& src, const Params& p, double t0) {
+  yaspmv_status st;
   if (A->device >= 0 && !find_kernel(A->dtype, p.h, p.w, p.T, p.col_mode, p.rc > 0 ? 2 : 1))
     return fail(YASPMV_EUNSUPPORTED, "no compiled kernel for this (dtype, h, w, T): values per thread > 512 B");
   if ((p.flags & YASPMV_GPU_ENCODE) && A->device >= 0) {
@@ -234,7 +390,7 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
     Canonical meta;
     GpuArrays g;
     int64_t esc = 0;
-    if ((st = encode_gpu(A->csr, p, meta, g, esc, nullptr)) != YASPMV_OK) return st;
+    if ((st = encode_gpu(src, p, meta, g, esc, nullptr)) != YASPMV_OK) return st;
     DevArrays nd;
     for (int r = 0; r < 4; ++r) nd.val[r] = g.val[r];
     nd.col = g.col;
@@ -268,7 +424,7 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
     return YASPMV_OK;
   }
   Canonical c;
-  if ((st = encode(A->csr, p, c)) != YASPMV_OK) return st;
+  if ((st = encode(src, p, c)) != YASPMV_OK) return st;
   if ((st = install_canonical_impl(A, std::move(c), p.flags)) != YASPMV_OK) return st;
   A->build_s = now_s() - t0;
   return YASPMV_OK;
@@ -306,6 +462,11 @@ int64_t format_bytes(const yaspmv_matrix A) {
   b += c.ntiles * (4 + 16 + (p.h > 1 ? 8 * (int64_t)p.h : 0) + 16);  // cta_seg0, status(+carry), carries, hand-off
   if (c.has_seg_row) b += c.n_stops * 4;                         // seg_row
   b += c.n_zero * 4;                                             // zero-fill list
+  if (A->band_on) {                                              // band stream + its aux (P1-P6)
+    const PanelCanonical& q = A->pan;
+    b += q.nband_pad * (int64_t)(A->vsize + 2) + q.nband_pad / 8;
+    b += (q.g.npanels + 1) * 8 + 2 * q.g.npanels * (q.g.KS + 1) * 4 + q.g.npanels * q.g.KS * q.g.nw() * 6;
+  }
   return b;
 }
 
@@ -313,16 +474,18 @@ int64_t alg_bytes(const yaspmv_matrix A) {
   const Canonical& c = A->can;
   const Params& p = c.p;
   int64_t b = format_bytes(A) + c.n * A->vsize;  // + x
+  if (A->band_on) b += c.m * A->vsize;           // + the band kernel's read of the far part's y
   if (p.S == 1) b += c.m * A->vsize;             // + y
   else b += (int64_t)p.S * c.MB * p.h * A->vsize + (int64_t)p.S * c.m * A->vsize + c.m * A->vsize;
   return b;
 }
 
-yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2 = nullptr,
-                       double* out_norm2 = nullptr, int ablate = 0, const PeerOut* peers = nullptr) {
+yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2,
+                             double* out_norm2, int ablate, const PeerOut* peers) {
   const Canonical& c = A->can;
   const Params& p = c.p;
   cudaStream_t cs = (cudaStream_t)stream;
+  DeviceGuard dg(A->device);  // the handle's device, whatever the caller's current one is
   if (c.m == 0) {
     if (out_norm2) CUDA_TRY(cudaMemsetAsync(out_norm2, 0, sizeof(double), cs));
     return YASPMV_OK;
@@ -380,6 +543,8 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   for (int q = 0; q < YASPMV_MAX_RANKS; ++q) a.peer_out[q] = nullptr;
   a.rcache = p.rc * p.C;
   a.tpc = A->tpc;
+  a.spin_limit = debug_spin_limit();
+  a.spin_tile = debug_spin_slot();
   if (ablate && p.rc > 0) return fail(YASPMV_EUNSUPPORTED, "ablation / probe variants are strategy-1 kernels");
   if (peers && p.S == 1) {  // S > 1: the kernel writes tmp, the combine writes the peers
     a.npeer = peers->n;
@@ -410,6 +575,52 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   }
   if (out_norm2) {
     launch_sum_f64(A->d_part, npart, out_norm2, A->d_scratch, stream);
+    CUDA_TRY(cudaGetLastError());
+  }
+  return YASPMV_OK;
+}
+
+// y := A x: the plain path, or for a panel-sliced BCCOO+ handle the far part (plain path,
+// y := A_far x) followed by the band kernel (y += slices, in order; epilogue on the result)
+yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2 = nullptr,
+                       double* out_norm2 = nullptr, int ablate = 0, const PeerOut* peers = nullptr) {
+  if (!A->band_on) return run_spmv_plain(A, x, y, stream, in_norm2, out_norm2, ablate, peers);
+  if (ablate || peers)
+    return fail(YASPMV_EUNSUPPORTED, "ablation variants and the fused exchange run the plain format only");
+  if (A->can.m == 0) {
+    if (out_norm2) CUDA_TRY(cudaMemsetAsync(out_norm2, 0, sizeof(double), (cudaStream_t)stream));
+    return YASPMV_OK;
+  }
+  DeviceGuard dg(A->device);
+  yaspmv_status st = run_spmv_plain(A, x, y, stream, nullptr, nullptr, 0, nullptr);
+  if (st != YASPMV_OK) return st;
+  const PanelGeom& g = A->pan.g;
+  PanelArgs pa;
+  pa.col16 = A->pd.col16;
+  pa.val = A->pd.val;
+  pa.flags = A->pd.flags;
+  pa.panel_blk0 = A->pd.panel_blk0;
+  pa.slice_ptr = A->pd.slice_ptr;
+  pa.stop_ptr = A->pd.stop_ptr;
+  pa.occ = A->pd.occ;
+  pa.pre = A->pd.pre;
+  pa.x = x;
+  pa.y = y;
+  pa.m = A->can.m;
+  pa.n = A->can.n;
+  pa.R = g.R;
+  pa.W = g.W;
+  pa.B = g.B;
+  pa.col0 = g.col0;
+  pa.KS = g.KS;
+  pa.npanels = g.npanels;
+  pa.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
+  pa.in_norm2 = in_norm2;
+  pa.part = A->pd.part;
+  const int e = launch_panel(pa, A->dtype, stream);
+  if (e != 0) return fail(YASPMV_ECUDA, std::string("panel kernel: ") + cudaGetErrorString((cudaError_t)e));
+  if (out_norm2) {
+    launch_sum_f64(A->pd.part, g.npanels, out_norm2, A->pd.scratch, stream);
     CUDA_TRY(cudaGetLastError());
   }
   return YASPMV_OK;
@@ -604,14 +815,15 @@ yaspmv_status yaspmv_host_sync(yaspmv_matrix A) {
 
 int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
   if (!A || A->can.m == 0) return 0;
-  if (A->can.ntiles == 0) return 0;  // memset only
-  return A->can.p.S > 1 ? 2 : 1;
+  const int band = A->band_on && A->pan.g.npanels > 0 ? 1 : 0;
+  if (A->can.ntiles == 0) return band;  // memset (+ the band kernel)
+  return (A->can.p.S > 1 ? 2 : 1) + band;
 }
 
 yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle");
-  if (variant < 1 || variant > 11) return fail(YASPMV_EINVAL, "ablation variant must be in 1..11");
+  if (variant < 1 || variant > 12) return fail(YASPMV_EINVAL, "ablation variant must be in 1..12");
   if (variant != 3 && (A->can.p.h != 1 || A->can.p.w != 1))
     return fail(YASPMV_EUNSUPPORTED, "ablation variants / probes are compiled for 1x1 blocks only");
   const int ab = variant == 1   ? ABL_DEFER_CARRY
@@ -624,6 +836,7 @@ yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void*
                  : variant == 9 ? (ABL_DEFER_CARRY | ABL_NO_FIXUP | ABL_NO_YSTORE)
                  : variant == 10 ? (ABL_STOP_SCAN | ABL_PROBE_PUB)
                  : variant == 11 ? (ABL_STOP_SCAN | ABL_PROBE_ST)
+                 : variant == 12 ? ABL_NO_PUBLISH0
                                  : 0;
   return run_spmv(A, x, y, stream, nullptr, nullptr, ab);
 }
@@ -648,7 +861,9 @@ yaspmv_status yaspmv_ablation_tree(const int32_t* rows, const uint8_t* flags, co
 }
 
 int32_t yaspmv_launches_per_power_step(yaspmv_matrix A) {
-  if (!A || A->can.m == 0 || A->can.ntiles == 0) return 0;
+  if (!A || A->can.m == 0) return 0;
+  if (A->band_on) return yaspmv_launches_per_spmv(A) + 2;  // far (+ combine) + band + the y^2 sum
+  if (A->can.ntiles == 0) return 0;
   return yaspmv_launches_per_spmv(A) + 2;  // + the two-level sum of the y^2 partials
 }
 
@@ -658,7 +873,7 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
   std::memset(o, 0, sizeof(*o));
   o->m = c.m;
   o->n = c.n;
-  o->nnz = c.nnz;
+  o->nnz = A->band_on ? A->nnz_total : c.nnz;
   o->MB = c.MB;
   o->NB = c.NB;
   o->SW = c.SW;
@@ -680,6 +895,13 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
   o->build_seconds = A->build_s;
   o->tune_seconds = A->tune_s;
   o->tune_candidates = A->tune_candidates;
+  if (A->band_on) {
+    o->band_blocks = A->pan.nband;
+    o->band_blocks_pad = A->pan.nband_pad;
+    o->band_panels = A->pan.g.npanels;
+    o->band_slices = A->pan.g.KS;
+    o->band_stops = A->pan.n_stops;
+  }
   return YASPMV_OK;
 }
 

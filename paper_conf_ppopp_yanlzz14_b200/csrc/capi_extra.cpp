@@ -42,6 +42,9 @@ struct ArrDesc {
   int ptb = 0;            // >0: stored permuted on the device with this per-thread byte run
   const void* host = nullptr;
   const void* dev = nullptr;
+  int64_t ntiles = -1;    // device layout tiles / threads (-1: the plain format's)
+  int C = 0;
+  bool band = false;      // a band-stream array (host copy: A->pan)
 };
 
 yaspmv_status describe(yaspmv_matrix A, int which, ArrDesc& d) {
@@ -104,8 +107,34 @@ yaspmv_status describe(yaspmv_matrix A, int which, ArrDesc& d) {
     case YASPMV_ARR_FRE:
       d.bytes = c.ntiles * p.C * 4;
       break;
-    default:
-      return fail(YASPMV_EINVAL, "unknown array id");
+    default: {
+      if (which < YASPMV_ARR_BAND_FLAGS || which > YASPMV_ARR_BAND_PRE) return fail(YASPMV_EINVAL, "unknown array id");
+      if (!A->band_on) return fail(YASPMV_EINVAL, "no band stream: the handle is not panel-sliced (band = 0)");
+      const PanelCanonical& q = A->pan;
+      const PanelGeom& g = q.g;
+      d.band = true;
+      d.ntiles = q.nband_pad / PANEL_TC;
+      d.C = PANEL_BC;
+      switch (which) {
+        case YASPMV_ARR_BAND_FLAGS:
+          d.bytes = q.nband_pad / 8; d.host = q.flags.data(); d.dev = A->pd.flags; break;
+        case YASPMV_ARR_BAND_COL16:
+          d.bytes = q.nband_pad * 2; d.host = q.col16.data(); d.dev = A->pd.col16; d.ptb = 2 * PANEL_BT; break;
+        case YASPMV_ARR_BAND_VAL:
+          d.bytes = q.nband_pad * A->vsize; d.host = q.val.data(); d.dev = A->pd.val; d.ptb = PANEL_BT * A->vsize;
+          break;
+        case YASPMV_ARR_BAND_PANEL_BLK0:
+          d.bytes = (g.npanels + 1) * 8; d.host = q.panel_blk0.data(); d.dev = A->pd.panel_blk0; break;
+        case YASPMV_ARR_BAND_SLICE_PTR:
+          d.bytes = g.npanels * (g.KS + 1) * 4; d.host = q.slice_ptr.data(); d.dev = A->pd.slice_ptr; break;
+        case YASPMV_ARR_BAND_STOP_PTR:
+          d.bytes = g.npanels * (g.KS + 1) * 4; d.host = q.stop_ptr.data(); d.dev = A->pd.stop_ptr; break;
+        case YASPMV_ARR_BAND_OCC:
+          d.bytes = g.npanels * g.KS * g.nw() * 4; d.host = q.occ.data(); d.dev = A->pd.occ; break;
+        default:
+          d.bytes = g.npanels * g.KS * g.nw() * 2; d.host = q.pre.data(); d.dev = A->pd.pre; break;
+      }
+    }
   }
   return YASPMV_OK;
 }
@@ -133,7 +162,7 @@ yaspmv_status yaspmv_export(yaspmv_matrix A, int32_t which, void* dst, int64_t b
     std::memcpy(dst, fre.data(), d.bytes);
     return YASPMV_OK;
   }
-  if (!A->have_host_arrays && which != YASPMV_ARR_CTA_SEG0)
+  if (d.band ? !A->have_pan_host : (!A->have_host_arrays && which != YASPMV_ARR_CTA_SEG0))
     return fail(YASPMV_EINVAL, "canonical host arrays released: build with YASPMV_KEEP_HOST");
   if (d.bytes) std::memcpy(dst, d.host, d.bytes);
   return YASPMV_OK;
@@ -167,7 +196,8 @@ yaspmv_status yaspmv_export_device(yaspmv_matrix A, int32_t which, void* dst, in
   } else {
     std::vector<uint8_t> tmp(d.bytes);
     CUDA_TRY(cudaMemcpy(tmp.data(), d.dev, d.bytes, cudaMemcpyDeviceToHost));
-    permute_from_device_layout(tmp.data(), static_cast<uint8_t*>(dst), c.ntiles, c.p.C, d.ptb);
+    permute_from_device_layout(tmp.data(), static_cast<uint8_t*>(dst), d.ntiles >= 0 ? d.ntiles : c.ntiles,
+                               d.ntiles >= 0 ? d.C : c.p.C, d.ptb);
   }
   return YASPMV_OK;
 }

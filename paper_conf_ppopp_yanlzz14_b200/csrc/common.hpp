@@ -28,13 +28,19 @@ enum Ablate {
   // with STOP_SCAN: after the scan, thread C-1 stores the tile's status word (PUB) / every
   // thread stores one value, coalesced (ST) — the cost of a CTA ending in stores
   ABL_PROBE_PUB = 512,
-  ABL_PROBE_ST = 1024
+  ABL_PROBE_ST = 1024,
+  // testing the debug spin bound: tile 0 never publishes its carry-out, so a look-back
+  // that reaches it polls forever (until YASPMV_SPIN_LIMIT traps)
+  ABL_NO_PUBLISH0 = 2048
 };
 
 struct Params {
   int h = 1, w = 1, S = 1, T = 16, C = 256, col_mode = 0, empty_mode = 0, flags = 0;
   int rc = 0;  // result cache size in units of C: 0 = strategy 1, k > 0 = strategy 2 (Table 1)
   int tpc = 0;  // tiles per CTA (0 = auto)
+  // panel-sliced BCCOO+ (panel.hpp): band half-width (0 = plain format), panel rows,
+  // slice width, column of row 0
+  int band = 0, pR = 0, pW = 0, col0 = 0;
 };
 
 inline int col_bytes(int mode) { return mode == COL_I32 ? 4 : 2; }
@@ -93,6 +99,8 @@ struct GpuArrays {
 // status helpers ------------------------------------------------------------------
 void set_error(const std::string& msg);
 yaspmv_status fail(yaspmv_status st, const std::string& msg);
+long long debug_spin_limit();   // YASPMV_SPIN_LIMIT (0 = unbounded look-back polling)
+long long* debug_spin_slot();   // mapped host slot for the trapped tile id (nullable)
 
 // encoder (encode.cpp) ---------------------------------------------------------------
 yaspmv_status normalize_csr(int64_t m, int64_t n, const int64_t* rp, const int32_t* ci, const void* v,
@@ -160,6 +168,10 @@ struct KArgs {
   void* peer_out[YASPMV_MAX_RANKS];
   int rcache;              // strategy 2: result cache entries (rc * C); 0 for strategy 1
   int tpc;                 // consecutive tiles per workgroup (block-id mode); grid = ceil(ntiles / tpc)
+  // debug spin bound: > 0 = a look-back that polls more than spin_limit times
+  // writes the waiting tile id to *spin_tile (mapped host memory) and traps
+  long long spin_limit;
+  long long* spin_tile;
 };
 
 // destinations of a fused exchange (combine kernel of BCCOO+, S > 1)

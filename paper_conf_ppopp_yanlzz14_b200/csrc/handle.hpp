@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include "common.hpp"
+#include "panel.hpp"
 
 using yaspmv::CSR;
 using yaspmv::Canonical;
@@ -65,6 +66,13 @@ struct yaspmv_matrix_s {
   int64_t n_escapes = 0;
   double build_s = 0, tune_s = 0;
   int tune_candidates = 0;
+  int64_t nnz_total = 0;          // structural non-zeros of A (far + band)
+  // panel-sliced BCCOO+ band part (params.band > 0); can/d then hold the far part
+  bool band_on = false;
+  yaspmv::PanelCanonical pan;     // host arrays (kept with YASPMV_KEEP_HOST / host-only)
+  yaspmv::PanelDev pd;
+  bool have_pan_host = false;
+  int pan_regs = 0;
   ~yaspmv_matrix_s() {
     if (device >= 0) {
       int cur = 0;
@@ -85,6 +93,7 @@ struct yaspmv_matrix_s {
       if (d_part) cudaFree(d_part);
       if (d_dep_row) cudaFree(d_dep_row);
       if (d_scratch) cudaFree(d_scratch);
+      pd.free_all();
       if (s_out) cudaStreamDestroy(s_out);
       cudaSetDevice(cur);
     }

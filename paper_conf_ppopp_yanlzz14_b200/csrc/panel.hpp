@@ -1,0 +1,101 @@
+// panel.hpp — the panel-sliced BCCOO+ part of an encoding (readings P1-P6).
+//
+// BCCOO+ (§2.3) stacks vertical slices of the matrix top-down so that
+// the rows of one slice share one part of x.  The panel variant does that inside
+// every horizontal panel of R rows, with slices of W columns placed relative to the panel
+// (column base cb(p) = p*R + col0 - B), so that one slice's part of x — W values — fits in
+// a CTA's shared memory and every gather of the slice is served from there instead of one
+// 32-byte L2 request per non-zero (profiles/r02_gather_microbench.md).  Entries outside
+// their panel's band [cb(p), cb(p) + KS*W) form an ordinary BCCOO matrix (the "far part",
+// encoded and run by the existing path).  y = A_far x, then each panel's slices in
+// ascending order add their segment sums (the BCCOO+ combine order, Q11) — in
+// shared memory, so BCCOO+'s temporary buffer never reaches HBM.
+#pragma once
+
+#include <cstdint>
+#include <vector>
+
+#include "../../include/yaspmv.h"
+
+namespace yaspmv {
+
+// band stream tile of the panel kernel: BT blocks per thread, BC threads per CTA
+constexpr int PANEL_BT = 16;
+constexpr int PANEL_BC = 512;
+constexpr int PANEL_TC = PANEL_BT * PANEL_BC;
+constexpr int PANEL_MAX_KS = 64;      // slices per panel
+constexpr int PANEL_NBUF = 3;         // x windows resident per CTA
+
+struct PanelGeom {
+  int64_t R = 0, W = 0, B = 0, col0 = 0;  // panel rows, slice width, band half-width, column of row 0
+  int64_t KS = 0;                         // slices per panel = ceil((R + 2B) / W)
+  int64_t npanels = 0;
+  int64_t nw() const { return R / 32; }   // bitmap words per slice
+};
+
+// host arrays (canonical layout, like Canonical for the plain format)
+struct PanelCanonical {
+  PanelGeom g;
+  int64_t nband = 0, nband_pad = 0, n_stops = 0;
+  std::vector<uint8_t> flags;       // nband_pad / 8, LSB-first, 0 = last entry of its row in its slice
+  std::vector<uint16_t> col16;      // nband_pad: column - cb(p) - k*W
+  std::vector<uint8_t> val;         // nband_pad values (raw bytes)
+  std::vector<int64_t> panel_blk0;  // npanels + 1
+  std::vector<int32_t> slice_ptr;   // npanels * (KS + 1)
+  std::vector<int32_t> stop_ptr;    // npanels * (KS + 1)
+  std::vector<uint32_t> occ;        // npanels * KS * nw
+  std::vector<uint16_t> pre;        // npanels * KS * nw
+  void release_arrays() {
+    std::vector<uint8_t>().swap(flags);
+    std::vector<uint16_t>().swap(col16);
+    std::vector<uint8_t>().swap(val);
+    std::vector<int64_t>().swap(panel_blk0);
+    std::vector<int32_t>().swap(slice_ptr);
+    std::vector<int32_t>().swap(stop_ptr);
+    std::vector<uint32_t>().swap(occ);
+    std::vector<uint16_t>().swap(pre);
+  }
+};
+
+struct PanelDev {
+  void* col16 = nullptr;        // device layout (tile transpose)
+  void* val = nullptr;          // device layout
+  uint8_t* flags = nullptr;     // canonical bit stream
+  int64_t* panel_blk0 = nullptr;
+  int32_t* slice_ptr = nullptr;
+  int32_t* stop_ptr = nullptr;
+  uint32_t* occ = nullptr;
+  uint16_t* pre = nullptr;
+  double* part = nullptr;       // per panel: sum of y^2 (power-iteration epilogue)
+  double* scratch = nullptr;
+  void free_all();
+};
+
+struct CSR;
+// split the normalised CSR A into the far part (owned CSR, all of A's rows) and the band
+// part (panel-sliced canonical arrays); R, W, B, col0 validated by the caller
+yaspmv_status encode_panel(const CSR& A, const PanelGeom& g, CSR& far, PanelCanonical& out);
+
+struct PanelArgs {
+  const void* col16;
+  const void* val;
+  const uint8_t* flags;
+  const int64_t* panel_blk0;
+  const int32_t* slice_ptr;
+  const int32_t* stop_ptr;
+  const uint32_t* occ;
+  const uint16_t* pre;
+  const void* x;
+  void* y;            // in: the far part's y; out: y = A x (scaled by the epilogue)
+  int64_t m, n;
+  int64_t R, W, B, col0, KS, npanels;
+  int epi;            // bit 0: scale by 1/sqrt(*in_norm2); bit 1: part[p] = sum over the panel of y^2
+  const double* in_norm2;
+  double* part;
+};
+// panel_kernel.cu
+int launch_panel(const PanelArgs& a, int dtype, void* stream);  // returns cudaError_t
+size_t panel_smem_bytes(int64_t R, int64_t W);
+int panel_attr(int64_t R, int64_t W, int* regs);                // cudaError_t; regs of the kernel
+
+}  // namespace yaspmv

@@ -238,12 +238,15 @@ struct ScanShared {
 // Warp-collective; waits only on predecessors nearer than that stop.  Polled with relaxed
 // loads (an acquire would invalidate L1 and with it the cached x); a carry value is read
 // only after its tile's epoch-tagged status word was seen (written before the release).
+// Forward progress rests on in-order dispatch or on ticket ids; a debug bound
+// (KArgs::spin_limit, YASPMV_SPIN_LIMIT) turns a hang into a trap naming the tile.
 template <int H>
 __device__ __forceinline__ void lookback(const KArgs& a, int64_t k, unsigned long long epoch, int lane,
                                          double (&carry)[H]) {
 #pragma unroll
   for (int r = 0; r < H; ++r) carry[r] = 0.0;
   int64_t jw = k - 1;
+  long long spins = 0;
   while (true) {
     const int64_t idx = jw - lane;
     int state = idx >= 0 ? 0 : 2;  // before tile 0: an inclusive prefix of 0
@@ -263,7 +266,15 @@ __device__ __forceinline__ void lookback(const KArgs& a, int64_t k, unsigned lon
         lim = p2 ? __ffs(p2) - 1 : 31;  // nearest tile with a row stop
         break;
       }
+      if (a.spin_limit > 0 && ++spins > a.spin_limit) {  // debug bound: report the tile, trap
+        if (lane == 0) *(volatile long long*)a.spin_tile = (long long)k;
+        __threadfence_system();
+        __trap();
+      }
     }
+    // h > 1: the carries are separate words written before a release of the status word;
+    // an acquire-release fence orders this warp's carry reads after the status reads
+    if constexpr (H > 1) asm volatile("fence.acq_rel.gpu;" ::: "memory");
 #pragma unroll
     for (int r = 0; r < H; ++r) {
       double cv = 0.0;
@@ -609,7 +620,8 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   // ---- step 3a: publish this tile's carry-out (adjacent sync) -----------
   bool succ_pending = false;
   unsigned long long succ_lo = 0, succ_hi = 0;
-  if (t == C - 1) publish_carry<VT, H, EPI>(a, tile, epoch, Fall, hs, acc, Vex, succ_pending, succ_lo, succ_hi);
+  if (t == C - 1 && !(EPI == 3 && (a.ablate & ABL_NO_PUBLISH0) && tile == 0))
+    publish_carry<VT, H, EPI>(a, tile, epoch, Fall, hs, acc, Vex, succ_pending, succ_lo, succ_hi);
 
   // ---- step 2c/3b: combine and write back -----------------------------
   const bool dependent = hs && !Fex && tile > 0;  // the tile's first stop needs the carry
@@ -1053,7 +1065,10 @@ int attr_spmv_s2(int C, int rc, int* regs, int* max_threads, int* blocks_per_sm)
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     if (dyn + fa.sharedSizeBytes > (size_t)optin) return 0;
     for (auto k : {k0, k1, k2}) {
-      e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+      // the cap is a property of the kernel instance, shared by every handle using it: set
+      // it to the opt-in limit once, never to this handle's size (a smaller later handle
+      // would otherwise lower it under an earlier handle's launches)
+      e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - (int)fa.sharedSizeBytes);
       if (e != cudaSuccess) return (int)e;
       e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 0);  // the rest stays L1
       if (e != cudaSuccess) return (int)e;

@@ -37,7 +37,8 @@ def _stream(stream) -> int | None:
 def make_params(**kw) -> _lib.Params:
     p = _lib.Params()
     names = {"h": "block_h", "w": "block_w", "S": "slices", "T": "thread_tile", "C": "cta_size",
-             "rc": "result_cache", "tpc": "tiles_per_cta"}
+             "rc": "result_cache", "tpc": "tiles_per_cta", "B": "band", "R": "panel_rows", "W": "slice_width",
+             "col0": "band_col0"}
     for k, v in kw.items():
         setattr(p, names.get(k, k), int(v))
     return p
@@ -159,10 +160,12 @@ class Matrix:
         return int(lib.yaspmv_launches_per_spmv(self._h))
 
     _ARR_DT = {"flags": np.uint8, "col_delta": np.int16, "seg_row": np.int32, "zero_rows": np.int32,
-               "cta_seg0": np.int32, "fre": np.int32}
+               "cta_seg0": np.int32, "fre": np.int32, "band_flags": np.uint8, "band_col16": np.uint16,
+               "band_panel_blk0": np.int64, "band_slice_ptr": np.int32, "band_stop_ptr": np.int32,
+               "band_occ": np.uint32, "band_pre": np.uint16}
 
     def _arr_dtype(self, name: str):
-        if name.startswith("val"):
+        if name.startswith("val") or name == "band_val":
             return self.dtype
         if name == "col":
             return np.uint16 if self.info()["params"]["col_mode"] == _lib.COL_U16 else np.int32
