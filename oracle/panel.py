@@ -14,16 +14,18 @@ of W columns placed relative to the panel (readings P1-P6):
       0 <= j - cb(p) < KS*W, else a FAR entry
   P3  band entries ordered by (p, k, i, j): the slices of a panel stacked top-down (the
       BCCOO+ rearrangement of P:150 inside the panel), every slice in BCCOO order (Fig. 2)
-  P4  bit flag 0 = last entry of row i inside slice (p, k); each panel padded with
-      '1' bits to a multiple of the workgroup tile T*C (pad entries: value 0 and the
-      stored column of the panel's last entry, as Q3 reads P:119 for plain BCCOO)
+  P4  bit flag 0 = last entry of row i inside slice (p, k); each slice (p, k) padded
+      with '1' bits to a multiple of the workgroup tile T*C (pad entries: value 0
+      and the stored column of the slice's last entry, as Q3 reads P:119 for plain BCCOO),
+      so that no workgroup tile holds two slices; empty slices hold no blocks
   P5  column stored as the unsigned short offset j - cb(p) - k*W  (< W <= 65536; the short
       column type of P:121/P:302 with a per-slice base, the original column = base +
       offset as P:150 requires)
   P6  rows of a slice without an entry hold no block; the slice's row-occupancy bitmap
       (R bits) maps the s-th row stop of the slice to the s-th set bit (the seg_row map of
-      reading Q1/R2, as a bitmap); per-word prefix counts and per-slice stop offsets
-      are aux arrays like cta_seg0
+      reading Q1/R2, as a bitmap); per-word prefix counts, per-slice stop offsets and,
+      per workgroup tile, the stops before it inside its slice (the first-result entry
+      of P:188-189, like cta_seg0) are aux arrays
   far entries: a plain BCCOO matrix of the same shape (encode.encode, E1-E9)
 
   y = A_far x  (O3 decode of the far part), then for every panel, slices in ascending k
@@ -46,7 +48,7 @@ class PanelParams:
     W: int = 8192         # slice width in columns (multiple of 4, <= 65536)
     B: int = 65536        # band half-width in columns
     T: int = 16           # band stream: blocks per thread
-    C: int = 512          # band stream: threads per workgroup
+    C: int = 32           # band stream: threads per workgroup tile (one warp)
     diag0: int = 0        # column of local row 0 (row-partitioned ranks: the rank's first row)
     far: E.Params = field(default_factory=E.Params)   # parameters of the far BCCOO part
 
@@ -64,10 +66,11 @@ class PanelEncoded:
     col16: np.ndarray       # uint16 [nband_pad]
     val: np.ndarray         # [nband_pad], dtype of A
     panel_blk0: np.ndarray  # int64 [npanels + 1]: first block of each panel
-    slice_ptr: np.ndarray   # int32 [npanels, KS + 1]: block offset of slice k inside its panel
+    slice_ptr: np.ndarray   # int32 [npanels, KS + 1]: block offset of slice k inside its panel (padded)
     stop_ptr: np.ndarray    # int32 [npanels, KS + 1]: row stops before slice k inside its panel
     occ: np.ndarray         # uint32 [npanels, KS, ceil(R / 32)]: row-occupancy bitmaps (LSB = lower row)
     pre: np.ndarray         # uint16 [npanels, KS, ceil(R / 32)]: set bits before each word
+    tile_rank: np.ndarray   # int32 [nband_pad / (T*C)]: stops before each tile inside its slice
     far: E.Encoded          # the far part (plain BCCOO)
     far_csr: tuple          # (row_ptr, col, val) of the far part
 
@@ -114,17 +117,21 @@ def encode_panel(m: int, n: int, row_ptr, col, val, pp: PanelParams) -> PanelEnc
     bp, bk, br, bc, bv = p[order], k[order], rows[order], col[order], val[order]
     nband = order.size
 
-    # per-panel block counts, padded to the workgroup tile
-    cnt = np.bincount(bp, minlength=npanels).astype(np.int64)
-    padded = -(-cnt // TC) * TC
+    # P4: every slice (p, k) padded to the workgroup tile; slices laid out in order
+    gcnt = np.zeros((npanels, KS), dtype=np.int64)
+    np.add.at(gcnt, (bp, bk), 1)
+    gpad = -(-gcnt // TC) * TC
+    slice_ptr = np.zeros((npanels, KS + 1), dtype=np.int64)
+    slice_ptr[:, 1:] = np.cumsum(gpad, axis=1)
     panel_blk0 = np.zeros(npanels + 1, dtype=np.int64)
-    np.cumsum(padded, out=panel_blk0[1:])
+    np.cumsum(slice_ptr[:, -1], out=panel_blk0[1:])
     nband_pad = int(panel_blk0[-1])
-    real0 = np.zeros(npanels + 1, dtype=np.int64)
-    np.cumsum(cnt, out=real0[1:])
-    pos = panel_blk0[bp] + (np.arange(nband) - real0[bp])      # stream position of each entry
+    gstart = np.zeros((npanels, KS), dtype=np.int64)       # first entry of each group in `order`
+    flat = np.cumsum(gcnt.ravel()) - gcnt.ravel()
+    gstart[:, :] = flat.reshape(npanels, KS)
+    pos = panel_blk0[bp] + slice_ptr[bp, bk] + (np.arange(nband) - gstart[bp, bk])
 
-    # P4: flags, 0 = last entry of its row inside its slice
+    # flags, 0 = last entry of its row inside its slice
     bits = np.ones(nband_pad, dtype=np.uint8)
     if nband:
         last = np.ones(nband, dtype=bool)
@@ -133,25 +140,22 @@ def encode_panel(m: int, n: int, row_ptr, col, val, pp: PanelParams) -> PanelEnc
         bits[pos[last]] = 0
     flags = np.packbits(bits, bitorder="little")
 
-    # P5: unsigned short column offset inside the slice
+    # P5: unsigned short column offset inside the slice; pad entries repeat the slice's
+    # last stored column (Q3)
     cb = bp * pp.R + pp.diag0 - pp.B
     col16 = np.zeros(nband_pad, dtype=np.uint16)
     col16[pos] = (bc - cb - bk * pp.W).astype(np.uint16)
-    for q in range(npanels):                    # pad entries repeat the panel's last column (Q3)
-        if cnt[q]:
-            last_pos = panel_blk0[q] + cnt[q] - 1
-            col16[last_pos + 1: panel_blk0[q + 1]] = col16[last_pos]
+    for q in range(npanels):
+        for kk in range(KS):
+            if gcnt[q, kk]:
+                last_pos = panel_blk0[q] + slice_ptr[q, kk] + gcnt[q, kk] - 1
+                col16[last_pos + 1: panel_blk0[q] + slice_ptr[q, kk + 1]] = col16[last_pos]
     vals = np.zeros(nband_pad, dtype=val.dtype)
     vals[pos] = bv
 
-    # P6: slice offsets, row-occupancy bitmaps, prefix counts, stop offsets
-    slice_ptr = np.zeros((npanels, KS + 1), dtype=np.int32)
+    # P6: row-occupancy bitmaps, prefix counts, stop offsets, stops before each tile
     occ_bits = np.zeros((npanels, KS, nw * 32), dtype=np.uint8)
-    for q in range(npanels):
-        sel = bp == q
-        kc = np.bincount(bk[sel], minlength=KS)
-        slice_ptr[q, 1:] = np.cumsum(kc)
-        occ_bits[q, bk[sel], br[sel] - q * pp.R] = 1
+    occ_bits[bp, bk, br - bp * pp.R] = 1
     occ = np.packbits(occ_bits.reshape(npanels, KS, nw, 32), axis=-1, bitorder="little")
     occ = occ.reshape(npanels, KS, nw, 4).copy().view("<u4").reshape(npanels, KS, nw).astype(np.uint32)
     wc = occ_bits.reshape(npanels, KS, nw, 32).sum(axis=-1)
@@ -159,8 +163,17 @@ def encode_panel(m: int, n: int, row_ptr, col, val, pp: PanelParams) -> PanelEnc
     pre[:, :, 1:] = np.cumsum(wc, axis=-1)[:, :, :-1]
     stop_ptr = np.zeros((npanels, KS + 1), dtype=np.int32)
     stop_ptr[:, 1:] = np.cumsum(wc.sum(axis=-1), axis=-1)
-    return PanelEncoded(m, n, pp, KS, npanels, nband, nband_pad, flags, col16, vals, panel_blk0, slice_ptr,
-                        stop_ptr, occ, pre, far, (frp, fcol, fval))
+    ntile = nband_pad // TC
+    tile_rank = np.zeros(ntile, dtype=np.int32)
+    stops_cum = np.zeros(nband_pad + 1, dtype=np.int64)
+    np.cumsum(1 - bits.astype(np.int64), out=stops_cum[1:])
+    for q in range(npanels):
+        for kk in range(KS):
+            g0 = panel_blk0[q] + slice_ptr[q, kk]
+            for tt in range(int(g0 // TC), int((panel_blk0[q] + slice_ptr[q, kk + 1]) // TC)):
+                tile_rank[tt] = stops_cum[tt * TC] - stops_cum[g0]
+    return PanelEncoded(m, n, pp, KS, npanels, nband, nband_pad, flags, col16, vals, panel_blk0,
+                        slice_ptr.astype(np.int32), stop_ptr, occ, pre, tile_rank, far, (frp, fcol, fval))
 
 
 def select_row(enc: PanelEncoded, q: int, k: int, s: int) -> int:
@@ -212,7 +225,10 @@ def to_dense(enc: PanelEncoded) -> np.ndarray:
         cb = q * pp.R + pp.diag0 - pp.B
         for k in range(enc.KS):
             s = 0
+            nst = int(enc.stop_ptr[q, k + 1] - enc.stop_ptr[q, k])
             for b in range(b0 + int(enc.slice_ptr[q, k]), b0 + int(enc.slice_ptr[q, k + 1])):
+                if s == nst:            # padding after the slice's last stop
+                    break
                 i = q * pp.R + select_row(enc, q, k, s)
                 d[i, cb + k * pp.W + int(enc.col16[b])] += float(enc.val[b])
                 s += bits[b] == 0

@@ -37,6 +37,7 @@ def test_hand_example_eq1_A():
     assert enc.slice_ptr.ravel().tolist() == g["slice_ptr"]
     assert enc.stop_ptr.ravel().tolist() == g["stop_ptr"]
     assert enc.occ.ravel().tolist() == g["occ"]
+    assert enc.tile_rank.tolist() == g["tile_rank"]
     assert enc.far_csr[2].tolist() == g["far_val"]
     x = np.arange(1, 9, dtype=np.float64)
     assert decode.spmv(enc.far, x).tolist() == g["y_far"]
@@ -60,6 +61,7 @@ def test_one_panel_one_slice_is_plain_bccoo(seed):
     assert np.array_equal(enc.flags, plain.flags)
     assert np.array_equal(enc.col16, plain.col)
     assert np.array_equal(enc.val, plain.val[0])
+    assert np.array_equal(enc.tile_rank, plain.cta_seg0)      # first-result entries
     rows_with = np.flatnonzero(np.diff(a.row_ptr) > 0)
     occ = np.unpackbits(enc.occ[0, 0].view(np.uint8), bitorder="little")[: a.m]
     assert np.array_equal(np.flatnonzero(occ), rows_with)
@@ -107,14 +109,22 @@ def test_invariants(seed):
     # every entry once: band + far = nnz; far entries lie outside their panel's band
     assert enc.nband == int(band.sum()) and enc.far_csr[1].size == a.nnz - enc.nband
     # stops = set bits of the occupancy bitmaps, slice by slice
+    TC = pp.T * pp.C
     for q in range(enc.npanels):
         b0 = enc.panel_blk0[q]
-        assert (enc.panel_blk0[q + 1] - b0) % (pp.T * pp.C) == 0
+        assert enc.panel_blk0[q + 1] - b0 == enc.slice_ptr[q, -1]
         for kk in range(enc.KS):
-            seg = bits[b0 + enc.slice_ptr[q, kk]: b0 + enc.slice_ptr[q, kk + 1]]
+            g0, g1 = b0 + enc.slice_ptr[q, kk], b0 + enc.slice_ptr[q, kk + 1]
+            assert g0 % TC == 0 and g1 % TC == 0               # no tile holds two slices (P4)
+            seg = bits[g0:g1]
             pops = sum(bin(int(w)).count("1") for w in enc.occ[q, kk])
             assert int((seg == 0).sum()) == pops == enc.stop_ptr[q, kk + 1] - enc.stop_ptr[q, kk]
-        assert np.all(bits[b0 + enc.slice_ptr[q, -1]: enc.panel_blk0[q + 1]] == 1)   # pad bits
+            if pops:
+                last = g0 + np.flatnonzero(seg == 0)[-1]
+                assert g1 - last - 1 < TC and np.all(bits[last + 1:g1] == 1)   # pad bits
+                assert np.all(enc.val[last + 1:g1] == 0)
+            for tt in range(g0 // TC, g1 // TC):               # first-result entry per tile
+                assert enc.tile_rank[tt] == int((bits[g0:tt * TC] == 0).sum())
     assert np.all(enc.col16.astype(np.int64) < pp.W)
     x = synth.make_x(a.n, np.float64, "int", seed)
     A = a.to_dense()
