@@ -36,7 +36,7 @@ def test_hand_example_eq1_A():
     assert enc.panel_blk0.tolist() == g["panel_blk0"]
     assert enc.slice_ptr.ravel().tolist() == g["slice_ptr"]
     assert enc.stop_ptr.ravel().tolist() == g["stop_ptr"]
-    assert enc.occ.ravel().tolist() == g["occ"]
+    assert enc.first_row.ravel().tolist() == g["first_row"] and enc.nfill == 0
     assert enc.tile_rank.tolist() == g["tile_rank"]
     assert enc.far_csr[2].tolist() == g["far_val"]
     x = np.arange(1, 9, dtype=np.float64)
@@ -50,23 +50,32 @@ def test_one_panel_one_slice_is_plain_bccoo(seed):
     """R >= m, B = 0, W >= R: every entry is a band entry of the single slice, and the
     band arrays are exactly the paper's BCCOO arrays (1x1 blocks, S = 1) with the seg_row
     reading (Q1/R2): same flags (P:114, P:119), columns (u16, P:302), values (P:105);
-    the occupancy bitmap marks exactly the rows of seg_row."""
+    and FILLER blocks exactly where the paper's reading R1 puts them."""
     a = synth.random_tiny(seed)
     R = 32 * (-(-a.m // 32))
     pp = PN.PanelParams(R=R, W=max(R, 4 * (-(-a.n // 4))), B=0, T=4, C=2)
     enc = PN.encode_panel(a.m, a.n, a.row_ptr, a.col, a.val, pp)
-    plain = E.encode(a.m, a.n, a.row_ptr, a.col, a.val, E.Params(1, 1, 1, 4, 2, E.COL_U16, E.EMPTY_MAP))
+    # the paper's arrays for the rows [first non-empty, last non-empty] with FILLER blocks
+    # (R1) for the empty rows in between; a filler's column is the zero slot W (Q3)
+    lens = np.diff(a.row_ptr)
+    nz = np.flatnonzero(lens > 0)
+    if nz.size == 0:
+        assert enc.nband_pad == 0
+        return
+    r0, r1 = nz[0], nz[-1] + 1
+    sub = synth.CSR(r1 - r0, a.n, a.row_ptr[r0:r1 + 1] - a.row_ptr[r0], a.col[a.row_ptr[r0]:a.row_ptr[r1]],
+                    a.val[a.row_ptr[r0]:a.row_ptr[r1]])
+    plain = E.encode(sub.m, sub.n, sub.row_ptr, sub.col, sub.val, E.Params(1, 1, 1, 4, 2, E.COL_U16, E.EMPTY_FILLER))
     assert enc.KS == 1 and enc.far.nnzb == 0 and enc.nband == a.nnz
+    assert enc.first_row[0, 0] == r0 and enc.nfill == plain.n_filler
     assert enc.nband_pad == plain.nnzb_pad
     assert np.array_equal(enc.flags, plain.flags)
-    assert np.array_equal(enc.col16, plain.col)
     assert np.array_equal(enc.val, plain.val[0])
     assert np.array_equal(enc.tile_rank, plain.cta_seg0)      # first-result entries (P:188-189)
-    rows_with = np.flatnonzero(np.diff(a.row_ptr) > 0)
-    occ = np.unpackbits(enc.occ[0, 0].view(np.uint8), bitorder="little")[: a.m]
-    assert np.array_equal(np.flatnonzero(occ), rows_with)
-    if plain.seg_row.size:
-        assert np.array_equal(plain.seg_row, rows_with)
+    fill = enc.col16 == pp.W
+    pcol = plain.col.astype(np.int64)
+    assert np.array_equal(enc.col16[~fill], pcol[~fill].astype(np.uint16))
+    assert np.all(pcol[fill] == plain.NB)                     # both name the zero column (Q3)
 
 
 def _banded(seed, m, n, band, extra=0.1):
@@ -117,15 +126,20 @@ def test_invariants(seed):
             g0, g1 = b0 + enc.slice_ptr[q, kk], b0 + enc.slice_ptr[q, kk + 1]
             assert g0 % TC == 0 and g1 % TC == 0               # no tile holds two slices (P4)
             seg = bits[g0:g1]
-            pops = sum(bin(int(w)).count("1") for w in enc.occ[q, kk])
+            # one stop per row from the slice's first to its last non-empty row (P6)
+            rows_k = np.unique(rows[band & (p == q) & (k == kk)] - q * pp.R)
+            pops = int(rows_k[-1] - rows_k[0] + 1) if rows_k.size else 0
             assert int((seg == 0).sum()) == pops == enc.stop_ptr[q, kk + 1] - enc.stop_ptr[q, kk]
+            if rows_k.size:
+                assert enc.first_row[q, kk] == rows_k[0]
             if pops:
                 last = g0 + np.flatnonzero(seg == 0)[-1]
                 assert g1 - last - 1 < TC and np.all(bits[last + 1:g1] == 1)   # pad bits
                 assert np.all(enc.val[last + 1:g1] == 0)
             for tt in range(g0 // TC, g1 // TC):               # first-result entry per tile
                 assert enc.tile_rank[tt] == int((bits[g0:tt * TC] == 0).sum())
-    assert np.all(enc.col16.astype(np.int64) < pp.W)
+    assert np.all(enc.col16.astype(np.int64) <= pp.W)            # W: a FILLER block's zero slot
+    assert enc.nfill == int(((enc.col16 == pp.W) & (enc.val == 0)).sum()) > 0
     x = synth.make_x(a.n, np.float64, "int", seed)
     A = a.to_dense()
     assert np.array_equal(PN.spmv(enc, x), A @ x)
