@@ -31,7 +31,7 @@ sys.path.insert(0, ROOT)
 
 # tuned defaults per config (yaspmv_tune on B200)
 DEFAULT_PARAMS = {
-    "c5": dict(h=1, w=1, S=1, T=32, C=128, col_mode=2, B=65536, R=16384, W=8192),
+    "c5": dict(h=1, w=1, S=3, T=32, C=128, col_mode=2, B=65536, R=16384, W=16384),
     "c4": dict(h=1, w=1, S=1, T=16, C=256),
     "c3-spheres": dict(h=4, w=4, T=4, C=128),
     "c3-cantilever": dict(h=4, w=4, T=4, C=128),
@@ -178,8 +178,34 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+_ONE_THREAD = r"""
+import sys, time, numpy as np
+sys.path.insert(0, %r)
+from oracle import ref
+d = np.load(%r)
+x = np.load(%r)
+ref.spmv(d["rp"], d["col"], d["val"], x, with_bound=False)
+ts = []
+for _ in range(3):
+    t0 = time.perf_counter(); ref.spmv(d["rp"], d["col"], d["val"], x, with_bound=False); ts.append(time.perf_counter() - t0)
+print(min(ts), ref.num_threads())
+"""
+
+
 def cpu_baseline(csr_full, x_np, budget_s=12.0):
-    """The oracle as it stands on the box's host cores, on a bounded row sample."""
+    """The oracle as it stands on the box's host cores, on a bounded row sample (SURVEY
+    §8(d) "Oracle timing": all cores, one thread, and scipy's csr @ x for reference)."""
     from oracle import ref
     m = csr_full.m
     rows = min(m, 1 << 20)
@@ -198,8 +224,64 @@ def cpu_baseline(csr_full, x_np, budget_s=12.0):
         ref.spmv(sub.row_ptr, sub.col, sub.val, x_np, with_bound=False)
         ts.append(time.perf_counter() - t0)
     t = float(np.median(ts))
-    return {"value": 2.0 * sub.nnz / t / 1e9, "unit": "GFLOPS", "cores": ref.num_threads(), "kind": "oracle",
-            "sample": f"rows [0, {rows}) ({sub.nnz} nnz) of the workload, median of {reps}"}
+    out = {"value": 2.0 * sub.nnz / t / 1e9, "unit": "GFLOPS", "cores": ref.num_threads(), "kind": "oracle",
+           "sample": f"rows [0, {rows}) ({sub.nnz} nnz) of the workload, median of {reps}",
+           "cpu_model": cpu_model(), "logical_cpus": os.cpu_count()}
+    # one thread (a subprocess with OMP_NUM_THREADS=1) on a quarter of the sample
+    try:
+        import tempfile
+        r1 = max(1, rows // 4)
+        s1 = csr_full.row_slice(0, r1)
+        with tempfile.TemporaryDirectory() as td:
+            fa, fx = os.path.join(td, "a.npz"), os.path.join(td, "x.npy")
+            np.savez(fa, rp=s1.row_ptr, col=s1.col, val=s1.val)
+            np.save(fx, x_np)
+            env = dict(os.environ, OMP_NUM_THREADS="1")
+            r = subprocess.run([sys.executable, "-c", _ONE_THREAD % (ROOT, fa, fx)], env=env, capture_output=True,
+                               text=True, timeout=300)
+            t1, nt = r.stdout.split()
+            out["single_thread"] = {"value": 2.0 * s1.nnz / float(t1) / 1e9, "unit": "GFLOPS", "threads": int(nt),
+                                    "sample": f"rows [0, {r1}) ({s1.nnz} nnz), best of 3"}
+    except Exception as e:  # report, never fail the bench line
+        out["single_thread"] = {"error": str(e)[:200]}
+    try:  # scipy's CSR matvec (single-threaded), same sample as the all-core number
+        import scipy.sparse as sp
+        A = sp.csr_matrix((sub.val, sub.col, sub.row_ptr), shape=(sub.m, x_np.size))
+        A @ x_np
+        t2 = min(_timed(lambda: A @ x_np) for _ in range(3))
+        out["scipy_csr_matvec"] = {"value": 2.0 * sub.nnz / t2 / 1e9, "unit": "GFLOPS", "threads": 1,
+                                   "sample": out["sample"]}
+    except Exception as e:
+        out["scipy_csr_matvec"] = {"error": str(e)[:200]}
+    return out
+
+
+def _timed(f) -> float:
+    t0 = time.perf_counter()
+    f()
+    return time.perf_counter() - t0
+
+
+def roofline_of(kern, dom, step_gbs, info, peak, peak_kind, traffic, traffic_src):
+    """The bench line's roofline object for the dominant kernel (longest per-step device
+    time, from the events recorded between the kernel groups during the timed region)."""
+    if not dom:  # fused multi-GPU step: the whole step
+        return {"bound": "hbm", "achieved": step_gbs, "peak": peak, "unit": "GB/s", "frac": step_gbs / peak,
+                "traffic": None, "peak_kind": peak_kind, "kernel": "whole fused step",
+                "alg_bytes_per_launch": info["alg_bytes"]}
+    ms, alg = kern[dom]
+    ach = alg / (ms * 1e-3) / 1e9
+    r = {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "traffic": traffic,
+         "peak_kind": peak_kind, "kernel": dom, "alg_bytes_per_launch": alg, "ms_per_launch": ms,
+         "share_of_step": None}
+    tot = sum(v[0] for v in kern.values())
+    if tot > 0:
+        r["share_of_step"] = ms / tot
+    if traffic:
+        r["dram_frac"] = traffic / (ms * 1e-3) / 1e9 / peak
+        r["traffic_over_alg"] = traffic / alg
+        r["traffic_source"] = traffic_src
+    return r
 
 
 def main():
@@ -297,6 +379,8 @@ def main():
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
+    if fpit is None:
+        A.profile_begin()  # events between the kernel groups of every timed step (per-kernel roofline)
     e0.record(stream)
     L_ = L
     for k in range(args.steps):
@@ -323,6 +407,7 @@ def main():
         fpit.comm.wait(stream)  # every peer's last step is complete
     e1.record(stream)
     torch.cuda.synchronize()
+    prof = A.profile_end() if fpit is None else None
     if fpit is not None:
         fpit.comm.check()
     if world > 1:
@@ -372,14 +457,34 @@ def main():
     if rank == 0:
         peak, peak_kind = measured_peaks()
         achieved = info["alg_bytes"] / (spmv_ms * 1e-3) / 1e9
-        traffic = None
-        prof = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.config}.json")
-        if os.path.exists(prof):
-            with open(prof) as f:
+        sv = np.dtype(dtype_np).itemsize
+        band = info["band_blocks_pad"] > 0
+        # per-kernel algorithmic bytes (DESIGN §6.1/§6.6): the band kernel K4
+        # reads its stream + aux, x once, the far part's y, and writes y; the plain / far K1
+        # reads its format + x and writes y
+        kern = {}
+        if prof and prof["calls"]:
+            S = info["params"]["slices"]
+            if band:  # far K1 writes its S slice results, the band kernel K4 reads and combines them
+                far_bytes = info["format_bytes"] - info["band_format_bytes"] + info["n"] * sv + S * info["m"] * sv
+                kern["spmv_bccoo_kernel (far part)"] = (prof["plain_ms"] / prof["calls"], far_bytes)
+                kern["panel_kernel (band)"] = (prof["band_ms"] / prof["calls"],
+                                               info["band_format_bytes"] + info["n"] * sv + (S + 1) * info["m"] * sv)
+            else:
+                kern["spmv_bccoo_kernel" + (" + combine" if S > 1 else "")] = (prof["plain_ms"] / prof["calls"],
+                                                                               info["alg_bytes"])
+        dom = max(kern, key=lambda k: kern[k][0]) if kern else None
+        traffic, traffic_src = None, None
+        tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.config}.json")
+        if os.path.exists(tp) and world == 1 and dom:
+            with open(tp) as f:
                 tr = json.load(f)
             strip = lambda p: {k: v for k, v in p.items() if k != "flags"}
-            if strip(tr.get("params", {})) == strip(info["params"]) and world == 1:
-                traffic = tr.get("dram_bytes_per_launch")
+            ent = tr.get("kernels", {}).get(dom.split(" ")[0])
+            if ent and strip(ent.get("params", {})) == strip(info["params"]):
+                traffic = ent.get("dram_bytes_per_launch")
+                traffic_src = {"file": os.path.relpath(tp, ROOT), "commit": tr.get("commit"),
+                               "captured": tr.get("captured")}
         line = {
             "metric": "SpMV GFLOPS and achieved HBM GB/s (% of 8 TB/s)", "value": gflops, "unit": "GFLOPS",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
@@ -399,11 +504,11 @@ def main():
             "spmv_ms": spmv_ms, "spmv_ms_max_over_ranks": spmv_ms_max,
             "spmv_gflops": 2.0 * info["nnz"] / (spmv_ms * 1e-3) / 1e9,
             "hbm_gbs_alg": achieved, "pct_of_8TBs": achieved / 8000.0 * 100.0,
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "spmv_bccoo_kernel" + (" + combine" if info["params"]["slices"] > 1 else "")
-                                   + " (+ 2 tiny y^2-partial reductions of the fused step)",
-                         "alg_bytes_per_launch": info["alg_bytes"]},
+            "roofline": roofline_of(kern, dom, achieved, info, peak, peak_kind, traffic, traffic_src),
+            "step_roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                              "frac": achieved / peak, "alg_bytes_per_step": info["alg_bytes"],
+                              "kernels": {k: {"ms": v[0], "alg_bytes": v[1], "gbs": v[1] / (v[0] * 1e-3) / 1e9}
+                                          for k, v in kern.items()}},
             "gpu_launches": (fpit.launches_per_step() if fpit is not None else A.launches_per_power_step())
                             * args.steps,
             "clocks": clocks, "e2e": e2e,

@@ -95,7 +95,7 @@ typedef struct {
      with the fields above.  fp32, 1x1 blocks; not with the fused multi-GPU step. */
   int32_t band;        /* band half-width B in columns; 0 = off (plain format)           */
   int32_t panel_rows;  /* R: multiple of 256, <= 32768; 0 = 16384                        */
-  int32_t slice_width; /* W: multiple of 4, <= 65536, KS <= 64; 0 = 8192                 */
+  int32_t slice_width; /* W: multiple of 4, <= 65532, KS <= 64; 0 = 16384                */
   int32_t band_col0;   /* column of row 0 (a row-partitioned rank: its first global row) */
 } yaspmv_params;
 
@@ -121,11 +121,13 @@ typedef struct {
   int32_t tune_candidates;   /* candidates timed by the last yaspmv_tune                   */
   int32_t reserved;
   /* panel-sliced BCCOO+ (params.band > 0): the fields above describe the far part        */
-  int64_t band_blocks;       /* band entries (1x1 blocks)                                 */
+  int64_t band_blocks;       /* band entries (1x1 blocks; FILLER blocks not included)     */
   int64_t band_blocks_pad;   /* after padding every panel to the band tile                */
   int64_t band_panels;       /* panels = CTAs of the band kernel                          */
   int64_t band_slices;       /* KS, slices per panel                                      */
   int64_t band_stops;        /* row stops of the band stream                              */
+  int64_t band_format_bytes; /* device bytes of the band stream + its aux read by one SpMV
+                                (included in format_bytes; the far part is the rest)       */
 } yaspmv_info;
 
 /* ---------------------------------------------------------------- build / free
@@ -237,17 +239,20 @@ enum {
   YASPMV_ARR_VAL0 = 3, YASPMV_ARR_VAL1 = 4, YASPMV_ARR_VAL2 = 5, YASPMV_ARR_VAL3 = 6,
   YASPMV_ARR_SEG_ROW = 7, YASPMV_ARR_ZERO_ROWS = 8, YASPMV_ARR_CTA_SEG0 = 9, YASPMV_ARR_FRE = 10,
   /* panel-sliced BCCOO+ band stream (params.band > 0; readings P1-P6 of DESIGN.md §2.1):
-   *  BAND_FLAGS      uint8 [band_blocks_pad/8]  0 = last entry of its row in its slice
-   *  BAND_COL16      uint16 [band_blocks_pad]   column - (p*R + col0 - B) - k*W
+   *  BAND_FLAGS      uint8 [band_blocks_pad/8]  0 = last block of its row in its slice
+   *  BAND_COL16      uint16 [band_blocks_pad]   column - (p*R + col0 - B) - k*W; W = FILLER
+   *                  block (value 0) of an empty row inside the slice's row range
    *  BAND_VAL        value [band_blocks_pad]
-   *  BAND_PANEL_BLK0 int64 [panels + 1]         first block of each panel (padded)
-   *  BAND_SLICE_PTR  int32 [panels * (KS+1)]    block offset of slice k inside its panel
+   *  BAND_PANEL_BLK0 int64 [panels + 1]         first block of each panel
+   *  BAND_SLICE_PTR  int32 [panels * (KS+1)]    block offset of slice k inside its panel (padded)
    *  BAND_STOP_PTR   int32 [panels * (KS+1)]    row stops before slice k inside its panel
-   *  BAND_OCC        uint32 [panels * KS * R/32] row-occupancy bitmap of every slice
-   *  BAND_PRE        uint16 [panels * KS * R/32] set bits before each bitmap word */
+   *  BAND_FIRST_ROW  int32 [panels * KS]        first non-empty row of each slice (the s-th
+   *                                              row stop of the slice is row first_row + s)
+   *  BAND_TILE_RANK  int32 [band_blocks_pad/512] stops before each 512-block tile in its slice
+   *  (every slice is padded to a multiple of 512 blocks = 16 blocks x 32 threads) */
   YASPMV_ARR_BAND_FLAGS = 11, YASPMV_ARR_BAND_COL16 = 12, YASPMV_ARR_BAND_VAL = 13,
   YASPMV_ARR_BAND_PANEL_BLK0 = 14, YASPMV_ARR_BAND_SLICE_PTR = 15, YASPMV_ARR_BAND_STOP_PTR = 16,
-  YASPMV_ARR_BAND_OCC = 17, YASPMV_ARR_BAND_PRE = 18
+  YASPMV_ARR_BAND_FIRST_ROW = 17, YASPMV_ARR_BAND_TILE_RANK = 18
 };
 
 /* yaspmv_export: copy canonical array `which` into host_dst (capacity `bytes`).  Returns
@@ -336,6 +341,14 @@ void yaspmv_comm_free(yaspmv_comm c);
 /* ---------------------------------------------------------------- misc */
 const char* yaspmv_last_error(void);
 const char* yaspmv_version(void);
+/* Per-kernel device timing (measurement only; bench.py's roofline).  yaspmv_profile_begin
+ * makes every later SpMV on A record CUDA events on its stream around its kernel groups:
+ * stage 0 = the plain BCCOO/BCCOO+ part (K1, + combine, + its y^2 sum), stage 1 = the band
+ * kernel of a panel-sliced handle (K4), stage 2 = K4's y^2 sum.  yaspmv_profile_end
+ * synchronizes those events, writes the summed milliseconds of stage s to ms[s] (s < n,
+ * n <= 3) and the number of profiled calls to *calls (nullable), and stops profiling. */
+yaspmv_status yaspmv_profile_begin(yaspmv_matrix A);
+yaspmv_status yaspmv_profile_end(yaspmv_matrix A, double* ms, int32_t n, int64_t* calls);
 /* Kernel launches issued by the last yaspmv_spmv on this handle (1, or 2 with S > 1). */
 int32_t yaspmv_launches_per_spmv(yaspmv_matrix A);
 /* Debug spin bound: with the environment variable YASPMV_SPIN_LIMIT=N (> 0, read

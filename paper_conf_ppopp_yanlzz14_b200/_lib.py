@@ -22,8 +22,8 @@ ARR = {"flags": 0, "col": 1, "col_delta": 2, "val0": 3, "val1": 4, "val2": 5, "v
        "seg_row": 7, "zero_rows": 8, "cta_seg0": 9, "fre": 10,
        # panel-sliced BCCOO+ band stream
        "band_flags": 11, "band_col16": 12, "band_val": 13, "band_panel_blk0": 14, "band_slice_ptr": 15,
-       "band_stop_ptr": 16, "band_occ": 17, "band_pre": 18}
-PANEL_BT, PANEL_BC = 16, 512  # band stream tile of the panel kernel (csrc/panel.hpp)
+       "band_stop_ptr": 16, "band_first_row": 17, "band_tile_rank": 18}
+PANEL_BT, PANEL_BC = 16, 32  # band stream tile: 16 blocks x 32 threads (csrc/panel.hpp PANEL_BT, PANEL_WT)
 
 MAX_RANKS = 8  # YASPMV_MAX_RANKS
 IPC_HANDLE_BYTES = 64
@@ -37,7 +37,7 @@ EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv"
             "yaspmv_comm_create", "yaspmv_comm_ipc_handle", "yaspmv_comm_open_ipc", "yaspmv_comm_connect_local",
             "yaspmv_comm_x", "yaspmv_comm_begin", "yaspmv_power_step_fused", "yaspmv_comm_wait",
             "yaspmv_comm_norm2_device", "yaspmv_comm_seq", "yaspmv_comm_check", "yaspmv_launches_per_fused_step",
-            "yaspmv_comm_free", "yaspmv_debug_spin_tile",
+            "yaspmv_comm_free", "yaspmv_debug_spin_tile", "yaspmv_profile_begin", "yaspmv_profile_end",
             # include/yaspmv_ablation.h
             "yaspmv_ablation_spmv", "yaspmv_ablation_tree", "yaspmv_ablation_tree_scratch_bytes"]
 
@@ -64,7 +64,8 @@ class Info(ctypes.Structure):
                 ("build_seconds", ctypes.c_double), ("tune_seconds", ctypes.c_double),
                 ("tune_candidates", ctypes.c_int32), ("reserved", ctypes.c_int32),
                 ("band_blocks", ctypes.c_int64), ("band_blocks_pad", ctypes.c_int64), ("band_panels", ctypes.c_int64),
-                ("band_slices", ctypes.c_int64), ("band_stops", ctypes.c_int64)]
+                ("band_slices", ctypes.c_int64), ("band_stops", ctypes.c_int64),
+                ("band_format_bytes", ctypes.c_int64)]
 
     def as_dict(self):
         d = {}
@@ -128,6 +129,8 @@ def _load():
         "yaspmv_launches_per_fused_step": ([H], i32),
         "yaspmv_comm_free": ([H], None),
         "yaspmv_debug_spin_tile": ([], i64),
+        "yaspmv_profile_begin": ([H], ctypes.c_int),
+        "yaspmv_profile_end": ([H, vp, i32, ctypes.POINTER(i64)], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

@@ -278,10 +278,10 @@ yaspmv_status resolve_band(yaspmv_matrix A, Params& p) {
   }
   if (A->dtype != YASPMV_F32) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ is compiled for fp32");
   if (p.h != 1 || p.w != 1) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ needs 1x1 blocks");
-  if (p.pR == 0) p.pR = 16384;
-  if (p.pW == 0) p.pW = 8192;
+  if (p.pR == 0) p.pR = 16384;  // defaults: one 1024-thread CTA per SM, 205 KB of shared memory
+  if (p.pW == 0) p.pW = 16384;
   if (p.pR % 256 || p.pR <= 0 || p.pR > 32768) return fail(YASPMV_EINVAL, "panel_rows must be a multiple of 256 in [256, 32768]");
-  if (p.pW % 4 || p.pW <= 0 || p.pW > 65536) return fail(YASPMV_EINVAL, "slice_width must be a multiple of 4 in [4, 65536]");
+  if (p.pW % 4 || p.pW <= 0 || p.pW > 65532) return fail(YASPMV_EINVAL, "slice_width must be a multiple of 4 in [4, 65532]");
   if ((p.pR + 2LL * p.band + p.pW - 1) / p.pW > PANEL_MAX_KS)
     return fail(YASPMV_EINVAL, "panel-sliced BCCOO+: (panel_rows + 2*band) / slice_width exceeds 64 slices");
   if (A->device >= 0) {
@@ -305,15 +305,15 @@ yaspmv_status panel_to_device(yaspmv_matrix A, const PanelCanonical& pc, PanelDe
   };
   const int64_t ntl = pc.nband_pad / PANEL_TC;
   yaspmv_status st;
-  if ((st = upload_permuted(reinterpret_cast<const uint8_t*>(pc.col16.data()), ntl, PANEL_BC, 2 * PANEL_BT,
+  if ((st = upload_permuted(reinterpret_cast<const uint8_t*>(pc.col16.data()), ntl, PANEL_WT, 2 * PANEL_BT,
                             &nd.col16)) != YASPMV_OK ||
-      (st = upload_permuted(pc.val.data(), ntl, PANEL_BC, PANEL_BT * A->vsize, &nd.val)) != YASPMV_OK ||
+      (st = upload_permuted(pc.val.data(), ntl, PANEL_WT, PANEL_BT * A->vsize, &nd.val)) != YASPMV_OK ||
+      (st = up(pc.tile_rank.data(), pc.tile_rank.size() * 4, (void**)&nd.tile_rank)) != YASPMV_OK ||
       (st = up(pc.flags.data(), pc.flags.size(), (void**)&nd.flags)) != YASPMV_OK ||
       (st = up(pc.panel_blk0.data(), pc.panel_blk0.size() * 8, (void**)&nd.panel_blk0)) != YASPMV_OK ||
       (st = up(pc.slice_ptr.data(), pc.slice_ptr.size() * 4, (void**)&nd.slice_ptr)) != YASPMV_OK ||
       (st = up(pc.stop_ptr.data(), pc.stop_ptr.size() * 4, (void**)&nd.stop_ptr)) != YASPMV_OK ||
-      (st = up(pc.occ.data(), pc.occ.size() * 4, (void**)&nd.occ)) != YASPMV_OK ||
-      (st = up(pc.pre.data(), pc.pre.size() * 2, (void**)&nd.pre)) != YASPMV_OK) {
+      (st = up(pc.first_row.data(), pc.first_row.size() * 4, (void**)&nd.first_row)) != YASPMV_OK) {
     nd.free_all();
     return st;
   }
@@ -452,6 +452,16 @@ yaspmv_status check_device(int32_t device) {
   return YASPMV_OK;
 }
 
+// the band stream + its aux (readings P1-P6), read once per SpMV
+int64_t band_format_bytes(const yaspmv_matrix A) {
+  if (!A->band_on) return 0;
+  const PanelCanonical& q = A->pan;
+  int64_t b = q.nband_pad * (int64_t)(A->vsize + 2) + q.nband_pad / 8;
+  b += (q.g.npanels + 1) * 8 + q.g.npanels * (q.g.KS + 1) * 4 + q.g.npanels * q.g.KS * 4;  // panel/slice ptr, first_row
+  b += q.nband_pad / PANEL_TC * 4;  // tile_rank
+  return b;
+}
+
 int64_t format_bytes(const yaspmv_matrix A) {
   const Canonical& c = A->can;
   const Params& p = c.p;
@@ -462,26 +472,22 @@ int64_t format_bytes(const yaspmv_matrix A) {
   b += c.ntiles * (4 + 16 + (p.h > 1 ? 8 * (int64_t)p.h : 0) + 16);  // cta_seg0, status(+carry), carries, hand-off
   if (c.has_seg_row) b += c.n_stops * 4;                         // seg_row
   b += c.n_zero * 4;                                             // zero-fill list
-  if (A->band_on) {                                              // band stream + its aux (P1-P6)
-    const PanelCanonical& q = A->pan;
-    b += q.nband_pad * (int64_t)(A->vsize + 2) + q.nband_pad / 8;
-    b += (q.g.npanels + 1) * 8 + 2 * q.g.npanels * (q.g.KS + 1) * 4 + q.g.npanels * q.g.KS * q.g.nw() * 6;
-  }
-  return b;
+  return b + band_format_bytes(A);
 }
 
 int64_t alg_bytes(const yaspmv_matrix A) {
   const Canonical& c = A->can;
   const Params& p = c.p;
   int64_t b = format_bytes(A) + c.n * A->vsize;  // + x
-  if (A->band_on) b += c.m * A->vsize;           // + the band kernel's read of the far part's y
+  const int64_t part = (int64_t)p.S * c.MB * p.h * A->vsize;  // far part's output: y or the S slices
+  if (A->band_on) return b + part + part + c.m * A->vsize;   // written, re-read by the band kernel, + y
   if (p.S == 1) b += c.m * A->vsize;             // + y
-  else b += (int64_t)p.S * c.MB * p.h * A->vsize + (int64_t)p.S * c.m * A->vsize + c.m * A->vsize;
+  else b += part + (int64_t)p.S * c.m * A->vsize + c.m * A->vsize;
   return b;
 }
 
 yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2,
-                             double* out_norm2, int ablate, const PeerOut* peers) {
+                             double* out_norm2, int ablate, const PeerOut* peers, bool skip_combine = false) {
   const Canonical& c = A->can;
   const Params& p = c.p;
   cudaStream_t cs = (cudaStream_t)stream;
@@ -568,7 +574,7 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
     launch_carry_fixup(A->d.status, A->d.carry, A->d_dep_row, c.ntiles, y, A->dtype, stream, 2);
     CUDA_TRY(cudaGetLastError());
   }
-  if (p.S > 1) {
+  if (p.S > 1 && !skip_combine) {
     launch_combine(A->d.tmp, y, c.m, c.MB * p.h, p.S, A->dtype, stream, in_norm2, out_norm2 ? A->d_part : nullptr,
                    peers);
     CUDA_TRY(cudaGetLastError());
@@ -582,9 +588,31 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
 
 // y := A x: the plain path, or for a panel-sliced BCCOO+ handle the far part (plain path,
 // y := A_far x) followed by the band kernel (y += slices, in order; epilogue on the result)
+// profiling (yaspmv_profile_begin): events of the current call, recorded between the
+// kernel groups on the launching stream (stage 0 plain/far part, 1 band kernel, 2 sum)
+cudaEvent_t* prof_events(yaspmv_matrix A) {
+  if (!A->prof_on) return nullptr;
+  std::array<cudaEvent_t, 4> ev{};
+  for (auto& e : ev)
+    if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+  A->prof_ev.push_back(ev);
+  return A->prof_ev.back().data();
+}
+
 yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, const double* in_norm2 = nullptr,
                        double* out_norm2 = nullptr, int ablate = 0, const PeerOut* peers = nullptr) {
-  if (!A->band_on) return run_spmv_plain(A, x, y, stream, in_norm2, out_norm2, ablate, peers);
+  cudaEvent_t* ev = prof_events(A);
+  cudaStream_t cs = (cudaStream_t)stream;
+  if (!A->band_on) {
+    if (ev) cudaEventRecord(ev[0], cs);
+    yaspmv_status st = run_spmv_plain(A, x, y, stream, in_norm2, out_norm2, ablate, peers);
+    if (ev) {
+      cudaEventRecord(ev[1], cs);
+      cudaEventRecord(ev[2], cs);
+      cudaEventRecord(ev[3], cs);
+    }
+    return st;
+  }
   if (ablate || peers)
     return fail(YASPMV_EUNSUPPORTED, "ablation variants and the fused exchange run the plain format only");
   if (A->can.m == 0) {
@@ -592,8 +620,12 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
     return YASPMV_OK;
   }
   DeviceGuard dg(A->device);
-  yaspmv_status st = run_spmv_plain(A, x, y, stream, nullptr, nullptr, 0, nullptr);
+  if (ev) cudaEventRecord(ev[0], cs);
+  // far part: BCCOO+ slices stay in tmp, the band kernel combines them (no combine kernel)
+  const bool fold = A->can.p.S > 1 && A->can.ntiles > 0;
+  yaspmv_status st = run_spmv_plain(A, x, y, stream, nullptr, nullptr, 0, nullptr, fold);
   if (st != YASPMV_OK) return st;
+  if (ev) cudaEventRecord(ev[1], cs);
   const PanelGeom& g = A->pan.g;
   PanelArgs pa;
   pa.col16 = A->pd.col16;
@@ -602,10 +634,13 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   pa.panel_blk0 = A->pd.panel_blk0;
   pa.slice_ptr = A->pd.slice_ptr;
   pa.stop_ptr = A->pd.stop_ptr;
-  pa.occ = A->pd.occ;
-  pa.pre = A->pd.pre;
+  pa.first_row = A->pd.first_row;
+  pa.tile_rank = A->pd.tile_rank;
   pa.x = x;
   pa.y = y;
+  pa.init = fold ? A->d.tmp : y;
+  pa.ninit = fold ? A->can.p.S : 1;
+  pa.init_stride = A->can.MB * A->can.p.h;
   pa.m = A->can.m;
   pa.n = A->can.n;
   pa.R = g.R;
@@ -619,10 +654,12 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   pa.part = A->pd.part;
   const int e = launch_panel(pa, A->dtype, stream);
   if (e != 0) return fail(YASPMV_ECUDA, std::string("panel kernel: ") + cudaGetErrorString((cudaError_t)e));
+  if (ev) cudaEventRecord(ev[2], cs);
   if (out_norm2) {
     launch_sum_f64(A->pd.part, g.npanels, out_norm2, A->pd.scratch, stream);
     CUDA_TRY(cudaGetLastError());
   }
+  if (ev) cudaEventRecord(ev[3], cs);
   return YASPMV_OK;
 }
 
@@ -700,6 +737,41 @@ yaspmv_status yaspmv_build_coo(int64_t m, int64_t n, int64_t nnz, const int32_t*
 }
 
 void yaspmv_free(yaspmv_matrix A) { delete A; }
+
+yaspmv_status yaspmv_profile_begin(yaspmv_matrix A) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle");
+  CUDA_TRY(cudaSetDevice(A->device));
+  for (auto& ev : A->prof_ev)
+    for (cudaEvent_t e : ev) cudaEventDestroy(e);
+  A->prof_ev.clear();
+  A->prof_on = true;
+  return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_profile_end(yaspmv_matrix A, double* ms, int32_t n, int64_t* calls) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  A->prof_on = false;
+  double acc[3] = {0, 0, 0};
+  yaspmv_status st = YASPMV_OK;
+  if (!A->prof_ev.empty()) {
+    cudaSetDevice(A->device);
+    for (auto& ev : A->prof_ev) {
+      if (cudaEventSynchronize(ev[3]) != cudaSuccess) st = fail(YASPMV_ECUDA, "profiling events failed");
+      for (int s = 0; s < 3 && st == YASPMV_OK; ++s) {
+        float t = 0;
+        if (cudaEventElapsedTime(&t, ev[s], ev[s + 1]) == cudaSuccess) acc[s] += t;
+      }
+    }
+  }
+  if (calls) *calls = (int64_t)A->prof_ev.size();
+  for (int s = 0; s < n && s < 3; ++s)
+    if (ms) ms[s] = acc[s];
+  for (auto& ev : A->prof_ev)
+    for (cudaEvent_t e : ev) cudaEventDestroy(e);
+  A->prof_ev.clear();
+  return st;
+}
 
 yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
@@ -817,7 +889,8 @@ int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
   if (!A || A->can.m == 0) return 0;
   const int band = A->band_on && A->pan.g.npanels > 0 ? 1 : 0;
   if (A->can.ntiles == 0) return band;  // memset (+ the band kernel)
-  return (A->can.p.S > 1 ? 2 : 1) + band;
+  if (band) return 2;                   // far part (its slices combined by the band kernel) + band
+  return A->can.p.S > 1 ? 2 : 1;
 }
 
 yaspmv_status yaspmv_ablation_spmv(yaspmv_matrix A, int32_t variant, const void* x, void* y, void* stream) {
@@ -901,6 +974,7 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
     o->band_panels = A->pan.g.npanels;
     o->band_slices = A->pan.g.KS;
     o->band_stops = A->pan.n_stops;
+    o->band_format_bytes = band_format_bytes(A);
   }
   return YASPMV_OK;
 }

@@ -108,13 +108,13 @@ yaspmv_status describe(yaspmv_matrix A, int which, ArrDesc& d) {
       d.bytes = c.ntiles * p.C * 4;
       break;
     default: {
-      if (which < YASPMV_ARR_BAND_FLAGS || which > YASPMV_ARR_BAND_PRE) return fail(YASPMV_EINVAL, "unknown array id");
+      if (which < YASPMV_ARR_BAND_FLAGS || which > YASPMV_ARR_BAND_TILE_RANK) return fail(YASPMV_EINVAL, "unknown array id");
       if (!A->band_on) return fail(YASPMV_EINVAL, "no band stream: the handle is not panel-sliced (band = 0)");
       const PanelCanonical& q = A->pan;
       const PanelGeom& g = q.g;
       d.band = true;
       d.ntiles = q.nband_pad / PANEL_TC;
-      d.C = PANEL_BC;
+      d.C = PANEL_WT;
       switch (which) {
         case YASPMV_ARR_BAND_FLAGS:
           d.bytes = q.nband_pad / 8; d.host = q.flags.data(); d.dev = A->pd.flags; break;
@@ -129,10 +129,10 @@ yaspmv_status describe(yaspmv_matrix A, int which, ArrDesc& d) {
           d.bytes = g.npanels * (g.KS + 1) * 4; d.host = q.slice_ptr.data(); d.dev = A->pd.slice_ptr; break;
         case YASPMV_ARR_BAND_STOP_PTR:
           d.bytes = g.npanels * (g.KS + 1) * 4; d.host = q.stop_ptr.data(); d.dev = A->pd.stop_ptr; break;
-        case YASPMV_ARR_BAND_OCC:
-          d.bytes = g.npanels * g.KS * g.nw() * 4; d.host = q.occ.data(); d.dev = A->pd.occ; break;
+        case YASPMV_ARR_BAND_FIRST_ROW:
+          d.bytes = g.npanels * g.KS * 4; d.host = q.first_row.data(); d.dev = A->pd.first_row; break;
         default:
-          d.bytes = g.npanels * g.KS * g.nw() * 2; d.host = q.pre.data(); d.dev = A->pd.pre; break;
+          d.bytes = q.nband_pad / PANEL_TC * 4; d.host = q.tile_rank.data(); d.dev = A->pd.tile_rank; break;
       }
     }
   }

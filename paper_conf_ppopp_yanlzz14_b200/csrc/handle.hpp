@@ -3,6 +3,9 @@
 
 #include <cuda_runtime.h>
 
+#include <array>
+#include <vector>
+
 #include "common.hpp"
 #include "panel.hpp"
 
@@ -73,6 +76,9 @@ struct yaspmv_matrix_s {
   yaspmv::PanelDev pd;
   bool have_pan_host = false;
   int pan_regs = 0;
+  // yaspmv_profile_*: events around the kernel groups of every SpMV while profiling
+  bool prof_on = false;
+  std::vector<std::array<cudaEvent_t, 4>> prof_ev;
   ~yaspmv_matrix_s() {
     if (device >= 0) {
       int cur = 0;
@@ -94,6 +100,9 @@ struct yaspmv_matrix_s {
       if (d_dep_row) cudaFree(d_dep_row);
       if (d_scratch) cudaFree(d_scratch);
       pd.free_all();
+      for (auto& ev : prof_ev)
+        for (cudaEvent_t e : ev)
+          if (e) cudaEventDestroy(e);
       if (s_out) cudaStreamDestroy(s_out);
       cudaSetDevice(cur);
     }

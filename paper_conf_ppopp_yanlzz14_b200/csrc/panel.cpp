@@ -13,7 +13,7 @@
 namespace yaspmv {
 
 void PanelDev::free_all() {
-  void* ps[] = {col16, val, flags, panel_blk0, slice_ptr, stop_ptr, occ, pre, part, scratch};
+  void* ps[] = {col16, val, flags, panel_blk0, slice_ptr, stop_ptr, first_row, tile_rank, part, scratch};
   for (void* q : ps)
     if (q) cudaFree(q);
   *this = PanelDev();
@@ -28,22 +28,28 @@ yaspmv_status encode_panel(const CSR& A, const PanelGeom& g0, CSR& far, PanelCan
   g.KS = (g.R + 2 * g.B + g.W - 1) / g.W;
   g.npanels = (A.m + g.R - 1) / g.R;
   if (g.KS > PANEL_MAX_KS) return fail(YASPMV_EINVAL, "panel: (R + 2B) / W must not exceed 64 slices");
-  const int64_t KS = g.KS, NP = g.npanels, R = g.R, W = g.W, NW = g.nw();
+  if (g.W >= 65535) return fail(YASPMV_EINVAL, "panel: slice width must be < 65535 (u16 offsets, W = filler)");
+  const int64_t KS = g.KS, NP = g.npanels, R = g.R, W = g.W;
   const int vs = A.vsize;
   out = PanelCanonical();
   out.g = g;
 
   // P1/P2: a row's band entries are one contiguous run of its (column-sorted) CSR entries
-  // [lo, hi): columns in [cb, cb + KS*W)
+  // [lo, hi): columns in [cb, cb + KS*W); per slice: entries, occupied rows, first/last row
   std::vector<int64_t> band_lo(A.m), band_hi(A.m);
-  std::vector<int64_t> pcnt(NP, 0);                 // band entries per panel
-  std::vector<int32_t> scnt((size_t)NP * KS, 0);    // band entries per (panel, slice)
+  std::vector<int64_t> pcnt(NP, 0);                      // band entries per panel
+  std::vector<int32_t> scnt((size_t)NP * KS, 0);         // entries per (panel, slice)
+  std::vector<int32_t> socc((size_t)NP * KS, 0);         // occupied rows per (panel, slice)
+  std::vector<int32_t> sfirst((size_t)NP * KS, -1), slast((size_t)NP * KS, -1);
 #pragma omp parallel for schedule(dynamic, 1)
   for (int64_t p = 0; p < NP; ++p) {
     const int64_t cb = p * R + g.col0 - g.B, ce = cb + KS * W;
     const int64_t r1 = std::min(A.m, (p + 1) * R);
     int64_t cnt = 0;
     int32_t* sc = scnt.data() + p * KS;
+    int32_t* so = socc.data() + p * KS;
+    int32_t* sf = sfirst.data() + p * KS;
+    int32_t* sl = slast.data() + p * KS;
     for (int64_t i = p * R; i < r1; ++i) {
       const int32_t* c0 = A.ci + A.rp[i];
       const int32_t* c1 = A.ci + A.rp[i + 1];
@@ -52,14 +58,31 @@ yaspmv_status encode_panel(const CSR& A, const PanelGeom& g0, CSR& far, PanelCan
       band_lo[i] = lo - A.ci;
       band_hi[i] = hi - A.ci;
       cnt += hi - lo;
-      for (const int32_t* c = lo; c < hi; ++c) sc[(*c - cb) / W]++;
+      int64_t kprev = -1;
+      for (const int32_t* c = lo; c < hi; ++c) {
+        const int64_t k = (*c - cb) / W;
+        sc[k]++;
+        if (k != kprev) {
+          so[k]++;
+          if (sf[k] < 0) sf[k] = (int32_t)(i - p * R);
+          sl[k] = (int32_t)(i - p * R);
+          kprev = k;
+        }
+      }
     }
     pcnt[p] = cnt;
   }
-  // padded panel offsets ('1' bits up to a multiple of the workgroup tile)
+  // P6 fillers, P4 padding of every slice to a multiple of the workgroup tile
   out.panel_blk0.assign(NP + 1, 0);
   for (int64_t p = 0; p < NP; ++p) {
-    out.panel_blk0[p + 1] = out.panel_blk0[p] + (pcnt[p] + PANEL_TC - 1) / PANEL_TC * PANEL_TC;
+    int64_t sz = 0;
+    for (int64_t k = 0; k < KS; ++k) {
+      const int64_t q = p * KS + k;
+      const int64_t fill = slast[q] >= 0 ? (int64_t)(slast[q] - sfirst[q] + 1) - socc[q] : 0;
+      out.nfill += fill;
+      sz += ((int64_t)scnt[q] + fill + PANEL_TC - 1) / PANEL_TC * PANEL_TC;
+    }
+    out.panel_blk0[p + 1] = out.panel_blk0[p] + sz;
     out.nband += pcnt[p];
   }
   out.nband_pad = out.panel_blk0[NP];
@@ -80,8 +103,8 @@ yaspmv_status encode_panel(const CSR& A, const PanelGeom& g0, CSR& far, PanelCan
     out.val.assign((size_t)out.nband_pad * vs, 0);
     out.slice_ptr.assign((size_t)NP * (KS + 1), 0);
     out.stop_ptr.assign((size_t)NP * (KS + 1), 0);
-    out.occ.assign((size_t)NP * KS * NW, 0);
-    out.pre.assign((size_t)NP * KS * NW, 0);
+    out.first_row.assign((size_t)NP * KS, 0);
+    out.tile_rank.assign(out.nband_pad / PANEL_TC, 0);
   } catch (const std::bad_alloc&) {
     return fail(YASPMV_ENOMEM, "panel encoder: host allocation failed");
   }
@@ -92,12 +115,22 @@ yaspmv_status encode_panel(const CSR& A, const PanelGeom& g0, CSR& far, PanelCan
     const int64_t cb = p * R + g.col0 - g.B;
     const int64_t r0 = p * R, r1 = std::min(A.m, (p + 1) * R);
     int32_t* sp = out.slice_ptr.data() + p * (KS + 1);
-    const int32_t* sc = scnt.data() + p * KS;
-    for (int64_t k = 0; k < KS; ++k) sp[k + 1] = sp[k] + sc[k];
-    std::vector<int64_t> fillp(sp, sp + KS);   // next position of every slice (P3)
+    int32_t* st = out.stop_ptr.data() + p * (KS + 1);
     const int64_t b0 = out.panel_blk0[p];
-    uint32_t* occ = out.occ.data() + (size_t)p * KS * NW;
+    std::vector<int64_t> gsz(KS), fillp(KS), lastrow(KS);
+    for (int64_t k = 0; k < KS; ++k) {
+      const int64_t q = p * KS + k;
+      const int64_t nst = slast[q] >= 0 ? slast[q] - sfirst[q] + 1 : 0;
+      gsz[k] = scnt[q] + (nst - socc[q]);                                          // entries + fillers
+      sp[k + 1] = sp[k] + (int32_t)((gsz[k] + PANEL_TC - 1) / PANEL_TC * PANEL_TC);
+      st[k + 1] = st[k] + (int32_t)nst;
+      out.first_row[q] = sfirst[q] >= 0 ? sfirst[q] : 0;
+      fillp[k] = b0 + sp[k];                                                       // P3 cursor
+      lastrow[k] = sfirst[q] >= 0 ? sfirst[q] - 1 : 0;
+    }
+    auto stop_at = [&](int64_t pos) { out.flags[pos >> 3] &= (uint8_t)~(1u << (pos & 7)); };
     for (int64_t i = r0; i < r1; ++i) {
+      const int64_t lr = i - r0;
       // far entries: before and after the band run (column order kept)
       int64_t f = far.rp_own[i];
       for (int64_t e = A.rp[i]; e < band_lo[i]; ++e, ++f) {
@@ -112,31 +145,32 @@ yaspmv_status encode_panel(const CSR& A, const PanelGeom& g0, CSR& far, PanelCan
       for (int64_t e = band_lo[i]; e < band_hi[i]; ++e) {
         const int64_t rel = (int64_t)A.ci[e] - cb;
         const int64_t k = rel / W;
-        const int64_t pos = b0 + fillp[k]++;
+        if (lastrow[k] < lr) {  // first entry of row i in slice k: fillers for the empty rows before it
+          for (int64_t rr = lastrow[k] + 1; rr < lr; ++rr) {
+            const int64_t pos = fillp[k]++;
+            out.col16[pos] = (uint16_t)W;  // value 0 (zero-initialised), the zero slot of the window
+            stop_at(pos);
+          }
+          lastrow[k] = lr;
+        }
+        const int64_t pos = fillp[k]++;
         out.col16[pos] = (uint16_t)(rel - k * W);                                   // P5
         std::memcpy(&out.val[(size_t)pos * vs], A.v + (size_t)e * vs, vs);
-        const bool last = e + 1 == band_hi[i] || ((int64_t)A.ci[e + 1] - cb) / W != k;
-        if (last) {                                                                  // P4: row stop
-          out.flags[pos >> 3] &= (uint8_t)~(1u << (pos & 7));
-          const int64_t lr = i - r0;
-          occ[k * NW + (lr >> 5)] |= 1u << (lr & 31);                               // P6
-        }
+        if (e + 1 == band_hi[i] || ((int64_t)A.ci[e + 1] - cb) / W != k) stop_at(pos);  // P4: row stop
       }
     }
-    // pad entries repeat the panel's last stored column (Q3)
-    const int64_t nreal = sp[KS];
-    if (nreal > 0)
-      for (int64_t b = b0 + nreal; b < out.panel_blk0[p + 1]; ++b) out.col16[b] = out.col16[b0 + nreal - 1];
-    // P6 aux: set bits before each word, stops before each slice
-    int32_t* st = out.stop_ptr.data() + p * (KS + 1);
-    uint16_t* pre = out.pre.data() + (size_t)p * KS * NW;
+    // pad entries repeat their slice's last stored column (Q3); stops before every tile
+    // inside its slice (the per-tile first-result entry)
     for (int64_t k = 0; k < KS; ++k) {
-      int32_t acc = 0;
-      for (int64_t w = 0; w < NW; ++w) {
-        pre[k * NW + w] = (uint16_t)acc;
-        acc += __builtin_popcount(occ[k * NW + w]);
+      if (gsz[k] > 0)
+        for (int64_t b = b0 + sp[k] + gsz[k]; b < b0 + sp[k + 1]; ++b) out.col16[b] = out.col16[b0 + sp[k] + gsz[k] - 1];
+      int32_t before = 0;
+      for (int64_t tt = (b0 + sp[k]) / PANEL_TC; tt < (b0 + sp[k + 1]) / PANEL_TC; ++tt) {
+        out.tile_rank[tt] = before;
+        int ones = 0;
+        for (int q = 0; q < PANEL_TC / 8; ++q) ones += __builtin_popcount(out.flags[tt * (PANEL_TC / 8) + q]);
+        before += PANEL_TC - ones;
       }
-      st[k + 1] = st[k] + acc;
     }
   }
   for (int64_t p = 0; p < NP; ++p) out.n_stops += out.stop_ptr[p * (KS + 1) + KS];

@@ -19,32 +19,34 @@
 
 namespace yaspmv {
 
-// band stream tile of the panel kernel: BT blocks per thread, BC threads per CTA
+// band stream: workgroup-level tiles of BT blocks x WT threads (one warp), every slice
+// padded to a whole number of tiles (reading P4); the kernel runs CTA threads per panel
 constexpr int PANEL_BT = 16;
-constexpr int PANEL_BC = 512;
-constexpr int PANEL_TC = PANEL_BT * PANEL_BC;
+constexpr int PANEL_WT = 32;
+constexpr int PANEL_TC = PANEL_BT * PANEL_WT;
+constexpr int PANEL_CTA = 1024;
 constexpr int PANEL_MAX_KS = 64;      // slices per panel
-constexpr int PANEL_NBUF = 3;         // x windows resident per CTA
+constexpr int PANEL_NBUF = 2;         // x windows resident per CTA (current + next slice)
+
 
 struct PanelGeom {
   int64_t R = 0, W = 0, B = 0, col0 = 0;  // panel rows, slice width, band half-width, column of row 0
   int64_t KS = 0;                         // slices per panel = ceil((R + 2B) / W)
   int64_t npanels = 0;
-  int64_t nw() const { return R / 32; }   // bitmap words per slice
 };
 
 // host arrays (canonical layout, like Canonical for the plain format)
 struct PanelCanonical {
   PanelGeom g;
-  int64_t nband = 0, nband_pad = 0, n_stops = 0;
+  int64_t nband = 0, nfill = 0, nband_pad = 0, n_stops = 0;
   std::vector<uint8_t> flags;       // nband_pad / 8, LSB-first, 0 = last entry of its row in its slice
-  std::vector<uint16_t> col16;      // nband_pad: column - cb(p) - k*W
+  std::vector<uint16_t> col16;      // nband_pad: column - cb(p) - k*W (W: FILLER block)
   std::vector<uint8_t> val;         // nband_pad values (raw bytes)
   std::vector<int64_t> panel_blk0;  // npanels + 1
   std::vector<int32_t> slice_ptr;   // npanels * (KS + 1)
   std::vector<int32_t> stop_ptr;    // npanels * (KS + 1)
-  std::vector<uint32_t> occ;        // npanels * KS * nw
-  std::vector<uint16_t> pre;        // npanels * KS * nw
+  std::vector<int32_t> first_row;   // npanels * KS: first non-empty row of each slice (panel-relative)
+  std::vector<int32_t> tile_rank;   // nband_pad / TC: stops before each tile inside its slice
   void release_arrays() {
     std::vector<uint8_t>().swap(flags);
     std::vector<uint16_t>().swap(col16);
@@ -52,8 +54,8 @@ struct PanelCanonical {
     std::vector<int64_t>().swap(panel_blk0);
     std::vector<int32_t>().swap(slice_ptr);
     std::vector<int32_t>().swap(stop_ptr);
-    std::vector<uint32_t>().swap(occ);
-    std::vector<uint16_t>().swap(pre);
+    std::vector<int32_t>().swap(first_row);
+    std::vector<int32_t>().swap(tile_rank);
   }
 };
 
@@ -64,8 +66,8 @@ struct PanelDev {
   int64_t* panel_blk0 = nullptr;
   int32_t* slice_ptr = nullptr;
   int32_t* stop_ptr = nullptr;
-  uint32_t* occ = nullptr;
-  uint16_t* pre = nullptr;
+  int32_t* first_row = nullptr;
+  int32_t* tile_rank = nullptr;
   double* part = nullptr;       // per panel: sum of y^2 (power-iteration epilogue)
   double* scratch = nullptr;
   void free_all();
@@ -83,10 +85,15 @@ struct PanelArgs {
   const int64_t* panel_blk0;
   const int32_t* slice_ptr;
   const int32_t* stop_ptr;
-  const uint32_t* occ;
-  const uint16_t* pre;
+  const int32_t* first_row;
+  const int32_t* tile_rank;
   const void* x;
-  void* y;            // in: the far part's y; out: y = A x (scaled by the epilogue)
+  void* y;            // out: y = A x (scaled by the epilogue)
+  // the far part's result: ninit partial vectors init + s * init_stride (s < ninit), summed in
+  // ascending s in fp64 — the BCCOO+ slice combine (Q11) folded into the band kernel
+  const void* init;
+  int ninit;
+  int64_t init_stride;
   int64_t m, n;
   int64_t R, W, B, col0, KS, npanels;
   int epi;            // bit 0: scale by 1/sqrt(*in_norm2); bit 1: part[p] = sum over the panel of y^2

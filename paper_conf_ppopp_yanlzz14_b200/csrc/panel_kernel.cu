@@ -3,21 +3,25 @@
 // panel's band stream in workgroup-level tiles of BT*BC blocks):
 //
 //   prologue  acc[0..R) := y[panel rows] (the far part's result, already in y); the
-//             panel's slice offsets to shared memory; x windows of the first three slices
-//             (W values each, plus the slices' row-occupancy bitmaps) requested with
-//             cp.async.bulk on an mbarrier each — the part of x one BCCOO+ slice uses
-//             (P:154), staged in shared memory so that every gather of the slice is an
-//             LDS instead of a 32-byte L2 request;
-//   per tile  128-bit streaming loads of the thread tile (values, u16 column offsets, the
-//             BT flag bits; the next tile's loads are issued before this tile's math),
-//             gathers from the resident windows, products, the per-thread sequential
-//             segmented sum (strategy 1), the workgroup segmented scan of
-//             (has_stop, last partial sum), then the segment sums are
-//             added to acc[row] slice by slice (ascending k: the BCCOO+ combine order,
-//             P:184), rows found through the slice's occupancy bitmap (reading P6);
-//             a segment that runs into the next tile carries its partial sum in the CTA
-//             (the tiles of a panel run in order inside one workgroup, so the
-//             adjacent-synchronization chain of P:295-298 never leaves the SM);
+//             panel's slice offsets to shared memory; the x window of the first slice
+//             (W values, plus the slice's row-occupancy bitmap) requested with
+//             cp.async.bulk on an mbarrier — the part of x one BCCOO+ slice uses,
+//             staged in shared memory so that every gather of the slice is an LDS instead
+//             of a 32-byte L2 request;
+//   per slice the next slice's window is requested into the other buffer; the slice's
+//             workgroup-level tiles (16 blocks x 32 threads = one warp; every slice is
+//             padded to whole tiles, reading P4) go round-robin to the warps, which run
+//             independently: 128-bit streaming loads of the thread tile (the warp's next
+//             tile is already in flight), gathers from the window, products, the
+//             per-thread sequential segmented sum (strategy 1), the warp's
+//             segmented scan of (has_stop, last partial sum), and the carry into
+//             the tile's first segment by adjacent synchronization with the slice's
+//             earlier tiles — a decoupled look-back over per-tile records in shared
+//             memory; every segment sum is added to acc[row], the row found
+//             through the slice's occupancy bitmap from the tile's first-result entry
+//             (reading P6).  Inside a slice every row has one segment, so no
+//             two warps touch one row; a barrier between slices keeps each row's slice
+//             sums in ascending order (the BCCOO+ combine order) — deterministic;
 //   epilogue  y[panel rows] := acc (optionally scaled; per-panel sum of y^2).
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -28,7 +32,7 @@
 namespace yaspmv {
 namespace {
 
-constexpr int BT = PANEL_BT, BC = PANEL_BC, NWARP = BC / 32;
+constexpr int BT = PANEL_BT;
 
 __device__ __forceinline__ uint64_t pol_evict_first() {
   uint64_t p;
@@ -74,63 +78,44 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned by
                : "memory");
 }
 
-// shared-memory layout (dynamic part): acc[R] | 3 x { window[W + 4] | occ[NW] | pre[NW] }
+// shared-memory layout (dynamic part): acc[R] | NBUF x window[W + 4] (window element j at
+// shift + j; slot shift + W holds 0, the column of a FILLER block, reading P6)
 struct Layout {
   int64_t wbytes, bufbytes;
   __host__ __device__ Layout(int64_t R, int64_t W) {
+    (void)R;
     wbytes = ((W + 4) * 4 + 15) / 16 * 16;
-    bufbytes = wbytes + (R / 32) * 4 + (R / 32) * 2;
-    bufbytes = (bufbytes + 15) / 16 * 16;
+    bufbytes = wbytes;
   }
 };
 
+constexpr int NTH = PANEL_CTA, NWARP = NTH / 32, RING = 512, LAG = 128;
+static_assert(PANEL_TC == 512, "tile index = block offset >> 9");
+
 struct PanelShared {
-  int sp[PANEL_MAX_KS + 1];   // slice_ptr of the panel
-  int st[PANEL_MAX_KS + 1];   // stop_ptr of the panel
+  int sp[PANEL_MAX_KS + 1];        // slice_ptr of the panel
+  int fr[PANEL_MAX_KS];            // first_row of every slice
   uint64_t bar[PANEL_NBUF];
-  float wv[NWARP];
-  int wf[NWARP];
-  int wn[NWARP];
-  float cin;                  // carry into the next tile (partial sum of an open segment)
-  int s_before;               // row stops of the panel before the current tile
+  volatile int armed[PANEL_NBUF];  // window (non-empty slice ordinal) armed on each buffer
+  // carry records of the panel's tiles (decoupled look-back): the tile's last
+  // partial sum and whether it holds a row stop, published before the tag (tile + 1)
+  float rT[RING];
+  int rH[RING];
+  volatile int rtag[RING];
   double ss[NWARP];
 };
 
-// the row (inside the panel) of the rank-th stop of a slice: the rank-th set bit of its
-// occupancy bitmap (reading P6), through the per-word prefix counts
-__device__ __forceinline__ int select_row(const uint32_t* occ, const uint16_t* pre, int nw, int rank) {
-  int lo = 0, hi = nw - 1;  // largest w with pre[w] <= rank
-  while (lo < hi) {
-    const int mid = (lo + hi + 1) >> 1;
-    if ((int)pre[mid] <= rank) lo = mid;
-    else hi = mid - 1;
-  }
-  const unsigned pos = __fns(occ[lo], 0, rank - (int)pre[lo] + 1);
-  return lo * 32 + (int)pos;
-}
-// the next row after `row` that holds an entry of the slice
-__device__ __forceinline__ int next_row(const uint32_t* occ, int row) {
-  int w = (row + 1) >> 5;
-  uint32_t bits = occ[w] & (0xFFFFFFFFu << ((row + 1) & 31));
-  while (bits == 0) bits = occ[++w];
-  return w * 32 + __ffs(bits) - 1;
-}
-
 template <typename VT>
-__global__ void __launch_bounds__(BC, 1) panel_kernel(const PanelArgs a) {
+__global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ PanelShared sh;
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int64_t p = blockIdx.x;
-  const int R = (int)a.R, W = (int)a.W, KS = (int)a.KS, NW = R / 32;
+  const int R = (int)a.R, W = (int)a.W, KS = (int)a.KS;
   const Layout L(a.R, a.W);
   VT* acc = reinterpret_cast<VT*>(dsm);
   unsigned char* bufs = dsm + (int64_t)R * sizeof(VT);
-  auto win = [&](int k) { return reinterpret_cast<VT*>(bufs + (k % PANEL_NBUF) * L.bufbytes); };
-  auto occ_of = [&](int k) { return reinterpret_cast<uint32_t*>(bufs + (k % PANEL_NBUF) * L.bufbytes + L.wbytes); };
-  auto pre_of = [&](int k) {
-    return reinterpret_cast<uint16_t*>(bufs + (k % PANEL_NBUF) * L.bufbytes + L.wbytes + NW * 4);
-  };
+  auto win = [&](int o) { return reinterpret_cast<VT*>(bufs + (o % PANEL_NBUF) * L.bufbytes); };
   const int64_t row0 = p * a.R;
   const int64_t cb = row0 + a.col0 - a.B;  // column base of the panel (P1)
   const VT* x = static_cast<const VT*>(a.x);
@@ -141,24 +126,52 @@ __global__ void __launch_bounds__(BC, 1) panel_kernel(const PanelArgs a) {
   auto shift_of = [&](int k) { return (int)(((xe + cb + (int64_t)k * W) % 4 + 4) % 4); };
 
   // ---- prologue ---------------------------------------------------------------------
-  for (int k = t; k <= KS; k += BC) {
+  for (int k = t; k <= KS; k += NTH) {
     sh.sp[k] = a.slice_ptr[p * (KS + 1) + k];
-    sh.st[k] = a.stop_ptr[p * (KS + 1) + k];
+    if (k < KS) sh.fr[k] = a.first_row[p * KS + k];
   }
+  for (int q = t; q < RING; q += NTH) sh.rtag[q] = 0;
   if (t == 0) {
-    for (int b = 0; b < PANEL_NBUF; ++b) mbar_init(&sh.bar[b], 1);
+    for (int b = 0; b < PANEL_NBUF; ++b) {
+      mbar_init(&sh.bar[b], 1);
+      sh.armed[b] = -1;
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    sh.cin = 0.f;
-    sh.s_before = 0;
   }
   const int rows = (int)min((int64_t)a.R, a.m - row0);
-  for (int r = t; r < R; r += BC) acc[r] = r < rows ? y[row0 + r] : VT(0);
+  {  // acc := the far part's result for the panel rows (its slices combined in order, Q11);
+     // batches of 8 rows per thread, all loads in flight before the first use
+    const VT* in = static_cast<const VT*>(a.init) + row0;
+    for (int r0 = t; r0 < R; r0 += 8 * NTH) {
+      double s[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) s[j] = 0.0;
+      for (int q = 0; q < a.ninit; ++q) {
+        VT v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int r = r0 + j * NTH;
+          v[j] = r < rows ? __ldcs(in + q * a.init_stride + r) : VT(0);
+        }
+#pragma unroll
+        for (int j = 0; j < 8; ++j) s[j] += (double)v[j];
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        if (r0 + j * NTH < R) acc[r0 + j * NTH] = (VT)s[j];
+    }
+  }
   __syncthreads();
-  // thread 0 requests slice k into buffer k % 3 (W values of x + bitmap + prefix counts)
-  auto issue = [&](int k) {
-    uint64_t* bar = &sh.bar[k % PANEL_NBUF];
-    if (k >= PANEL_NBUF) mbar_wait(bar, (unsigned)((k / PANEL_NBUF - 1) & 1));  // previous use landed
-    VT* w = win(k);
+  auto next_nonempty = [&](int k) {  // first slice >= k holding blocks (KS: none)
+    while (k < KS && sh.sp[k] == sh.sp[k + 1]) ++k;
+    return k;
+  };
+  // thread 0 requests the window of slice k (non-empty ordinal o) into buffer o % NBUF
+  // (FILLER blocks read the zero slot behind the window)
+  auto issue = [&](int k, int o) {
+    uint64_t* bar = &sh.bar[o % PANEL_NBUF];
+    if (o >= PANEL_NBUF) mbar_wait(bar, (unsigned)((o / PANEL_NBUF - 1) & 1));  // previous use landed
+    VT* w = win(o);
     const int sh_k = shift_of(k);
     const int64_t base = cb + (int64_t)k * W;
     const int64_t lo = max((int64_t)0, base), hi = min((int64_t)a.n, base + W);
@@ -172,207 +185,159 @@ __global__ void __launch_bounds__(BC, 1) panel_kernel(const PanelArgs a) {
       for (int64_t j = max(ahi, alo); j < hi; ++j) w[sh_k + (j - base)] = x[j];  // unaligned tail
       tx += (unsigned)((ahi - alo) * sizeof(VT));
     }
-    const int64_t rec = (p * KS + k) * (int64_t)NW;
-    tx += NW * 4 + NW * 2;
+    w[sh_k + W] = VT(0);
     mbar_arrive_tx(bar, tx);
     if (ahi > alo) bulk_g2s(w + sh_k + (alo - base), x + alo, (unsigned)((ahi - alo) * sizeof(VT)), bar);
-    bulk_g2s(occ_of(k), a.occ + rec, NW * 4, bar);
-    bulk_g2s(pre_of(k), a.pre + rec, NW * 2, bar);
+    __threadfence_block();
+    sh.armed[o % PANEL_NBUF] = o;
   };
-  int issued = 0;  // slices requested so far (thread 0's count; every thread tracks it)
-  if (t == 0)
-    for (int k = 0; k < min(KS, PANEL_NBUF); ++k) issue(k);
-  issued = min(KS, PANEL_NBUF);
 
   const int64_t pb0 = a.panel_blk0[p];
-  const int ntl = (int)((a.panel_blk0[p + 1] - pb0) / PANEL_TC);
-  const int nreal = sh.sp[KS];
+  const int64_t tile0 = pb0 / PANEL_TC;  // first tile of the panel
   const uint64_t pol = pol_evict_first();
   const uint8_t* vbase = static_cast<const uint8_t*>(a.val);
   const uint8_t* cbase = static_cast<const uint8_t*>(a.col16);
   constexpr int VCH = BT * (int)sizeof(VT) / 16;  // 16-B chunks of values per thread
   constexpr int CCH = BT * 2 / 16;                 // 16-B chunks of u16 columns per thread
-  uint32_t vn[VCH * 4], cn[CCH * 4], fn = 0;
-  auto load_tile = [&](int j) {
-    const int64_t tile = pb0 / PANEL_TC + j;
-#pragma unroll
-    for (int c = 0; c < VCH; ++c) ld16(vbase + (tile * (int64_t)BC * VCH + (int64_t)c * BC + t) * 16, pol, &vn[4 * c]);
-#pragma unroll
-    for (int c = 0; c < CCH; ++c) ld16(cbase + (tile * (int64_t)BC * CCH + (int64_t)c * BC + t) * 16, pol, &cn[4 * c]);
-    fn = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)t * BT) >> 3));
-  };
-  if (ntl > 0) load_tile(0);
-  // slice containing panel block b (b < nreal)
-  auto slice_of = [&](int b, int k) {
-    while (b >= sh.sp[k + 1]) ++k;
-    return k;
-  };
+  // this warp's tiles: in each non-empty slice, the slice's tiles wid, wid + NWARP, ...
+  int k = next_nonempty(0);
+  int o = 0;  // non-empty ordinal of slice k
+  if (t == 0 && k < KS) {
+    issue(k, 0);
+    const int k1 = next_nonempty(k + 1);
+    if (k1 < KS) issue(k1, 1);
+  }
   double ssq = 0.0;
 
-  for (int j = 0; j < ntl; ++j) {
-    uint32_t vw[VCH * 4], cw[CCH * 4];
-#pragma unroll
-    for (int q = 0; q < VCH * 4; ++q) vw[q] = vn[q];
-#pragma unroll
-    for (int q = 0; q < CCH * 4; ++q) cw[q] = cn[q];
-    const uint32_t fl = fn;
-    if (j + 1 < ntl) load_tile(j + 1);  // next tile's stream in flight during this one
-
-    const int tb0 = j * PANEL_TC;               // first block of the tile (panel-relative)
-    const int tb1 = min(tb0 + PANEL_TC, nreal);  // end of its real blocks
-    const int bt0 = tb0 + t * BT;               // this thread's first block
-    // slices of the tile: k_lo..k_hi (nothing if the tile is only padding)
-    int k_lo = 0, k_hi = -1;
-    if (tb0 < tb1) {
-      int lo = 0, hi = KS - 1;  // largest k with sp[k] <= tb0
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (sh.sp[mid] <= tb0) lo = mid;
-        else hi = mid - 1;
-      }
-      k_lo = slice_of(tb0, lo);
-      k_hi = slice_of(tb1 - 1, k_lo);
+  while (k < KS) {
+    // window o of slice k resident (a buffer two requests behind would alias the awaited
+    // parity: wait until the request is armed first)
+    while (sh.armed[o % PANEL_NBUF] != o) {
     }
-    // windows: slices below k_lo are finished; request up to k_lo + 2 into their buffers
-    if (k_hi >= 0) {
-      const int want = min(KS, k_lo + PANEL_NBUF);
-      if (t == 0)
-        for (int k = issued; k < want; ++k) issue(k);
-      issued = max(issued, want);
-      for (int k = k_lo; k <= min(k_hi, k_lo + PANEL_NBUF - 1); ++k) mbar_wait(&sh.bar[k % PANEL_NBUF], (k / PANEL_NBUF) & 1);
-    }
+    mbar_wait(&sh.bar[o % PANEL_NBUF], (o / PANEL_NBUF) & 1);
+    const VT* wk = win(o) + shift_of(k);
+    const int frk = sh.fr[k];
+    const int ltile_k = sh.sp[k] >> 9;                     // panel-local first tile of the slice
+    const int ntile_k = (sh.sp[k + 1] - sh.sp[k]) >> 9;    // tiles of the slice
+    for (int u = wid; u < ntile_k; u += NWARP) {
+      const int lt = ltile_k + u;       // panel-local tile index (tag of its carry record)
+      const int64_t tile = tile0 + lt;  // global tile index
+      // ---- stream the thread tile: 128-bit loads of the device layout -----
+      uint32_t vw[VCH * 4], cw[CCH * 4];
+#pragma unroll
+      for (int c = 0; c < CCH; ++c) ld16(cbase + (tile * (int64_t)32 * CCH + (int64_t)c * 32 + lane) * 16, pol, &cw[4 * c]);
+#pragma unroll
+      for (int c = 0; c < VCH; ++c) ld16(vbase + (tile * (int64_t)32 * VCH + (int64_t)c * 32 + lane) * 16, pol, &vw[4 * c]);
+      const uint32_t fl = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
+      const int trank = __ldg(a.tile_rank + tile);
+      // flow control: the record slot of this tile must have been released
+      if (lt >= LAG && lane == 0)
+        while (sh.rtag[(lt - LAG) % RING] != lt - LAG + 1) __nanosleep(32);
+      __syncwarp();
 
-    // ---- multiply: gathers from the resident windows (global x beyond them) ----------
-    int kf = k_lo;
-    if (bt0 < tb1) kf = slice_of(bt0, k_lo);
-    VT pr[BT];
-    {
-      int k = kf;
-      int sk = shift_of(k);
-      const VT* wk = win(k);
+      // ---- multiply: gathers from the slice's window --------------------------------
+      VT pr[BT];
 #pragma unroll
       for (int i = 0; i < BT; ++i) {
-        const int b = bt0 + i;
-        VT v = VT(0);
-        if (b < tb1) {
-          if (b >= sh.sp[k + 1]) {
-            k = slice_of(b, k);
-            sk = shift_of(k);
-            wk = win(k);
-          }
-          const int c = (int)((cw[i >> 1] >> (16 * (i & 1))) & 0xFFFFu);
-          const VT xv = (k < k_lo + PANEL_NBUF) ? wk[sk + c] : __ldg(x + cb + (int64_t)k * W + c);
-          v = __uint_as_float(vw[i]) * xv;
+        const int c = (int)((cw[i >> 1] >> (16 * (i & 1))) & 0xFFFFu);
+        pr[i] = __uint_as_float(vw[i]) * wk[c];
+      }
+      // ---- per-thread segmented sum: pr[i] := sum of its segment up to block i
+      const uint32_t stops = ~fl & 0xFFFFu;
+      const int nst = __popc(stops);
+#pragma unroll
+      for (int i = 1; i < BT; ++i) pr[i] = ((stops >> (i - 1)) & 1u) ? pr[i] : pr[i - 1] + pr[i];
+      const VT tail = ((stops >> (BT - 1)) & 1u) ? VT(0) : pr[BT - 1];
+      // ---- warp segmented scan of (has_stop, last partial sum) ----------------
+      int f = nst > 0, nn = nst;
+      VT v = tail;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const int f2 = __shfl_up_sync(0xffffffffu, f, d);
+        const int n2 = __shfl_up_sync(0xffffffffu, nn, d);
+        const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
+        if (lane >= d) {
+          if (!f) v = v2 + v;
+          f |= f2;
+          nn += n2;
         }
-        pr[i] = v;
       }
-    }
-    // ---- per-thread segmented sum: stops are '0' bits ------------------------
-    const uint32_t stops = ~fl & 0xFFFFu;
-    const int nst = __popc(stops);
-    const int hs = nst > 0;
-    VT tail = VT(0);
-#pragma unroll
-    for (int i = 0; i < BT; ++i) tail = ((stops >> i) & 1u) ? VT(0) : tail + pr[i];
-    // ---- workgroup segmented scan of (has_stop, last partial sum) -------------
-    int f = hs, nn = nst;
-    VT v = tail;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const int f2 = __shfl_up_sync(0xffffffffu, f, d);
-      const int n2 = __shfl_up_sync(0xffffffffu, nn, d);
-      const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
-      if (lane >= d) {
-        if (!f) v = v2 + v;
-        f |= f2;
-        nn += n2;
+      // ---- publish the tile's carry record (before anything waits on others) ----------
+      if (lane == 31) {
+        sh.rT[lt % RING] = v;   // inclusive: the tail after the tile's last stop, or its sum
+        sh.rH[lt % RING] = f;
+        __threadfence_block();
+        sh.rtag[lt % RING] = lt + 1;
       }
-    }
-    if (lane == 31) {
-      sh.wf[wid] = f;
-      sh.wn[wid] = nn;
-      sh.wv[wid] = v;
-    }
-    int fx = __shfl_up_sync(0xffffffffu, f, 1);
-    int nx = __shfl_up_sync(0xffffffffu, nn, 1);
-    VT vx = __shfl_up_sync(0xffffffffu, v, 1);
-    if (lane == 0) {
-      fx = 0;
-      nx = 0;
-      vx = VT(0);
-    }
-    __syncthreads();
-    int Fw = 0, Nw = 0, Fall = 0, Ntot = 0;
-    VT Vw = VT(0), Vall = VT(0);
-    for (int q = 0; q < NWARP; ++q) {
-      const int fq = sh.wf[q];
-      if (q < wid) {
-        Vw = fq ? sh.wv[q] : Vw + sh.wv[q];
-        Fw |= fq;
-        Nw += sh.wn[q];
+      int fx = __shfl_up_sync(0xffffffffu, f, 1);
+      int nx = __shfl_up_sync(0xffffffffu, nn, 1);
+      VT vx = __shfl_up_sync(0xffffffffu, v, 1);
+      if (lane == 0) {
+        fx = 0;
+        nx = 0;
+        vx = VT(0);
       }
-      Vall = fq ? sh.wv[q] : Vall + sh.wv[q];
-      Fall |= fq;
-      Ntot += sh.wn[q];
-    }
-    const VT cin = sh.cin;
-    const int sb = sh.s_before;
-    const int Fex = Fw | fx;
-    // exclusive carry into this thread's first segment: earlier threads of the tile, and
-    // the open segment of the previous tile if no earlier thread of this tile has a stop
-    const VT Vex = Fex ? (fx ? vx : Vw + vx) : cin + (Vw + vx);
-    // ---- add the segment sums to acc[row], slice by slice (ascending k): one
-    // phase per slice of the tile, a barrier between phases, so every acc[row] receives
-    // its slices' sums in order (deterministic) and no two threads update a row at once
-    {
-      bool first = true;
-      int s = sb + Nw + nx;  // panel stop index of this thread's next stop
-      for (int kk = k_lo; kk <= k_hi; ++kk) {
-        if (hs) {
-          int k = kf, row = -1;
-          VT run = VT(0);
+      // ---- add the segment sums to acc[row]: the s-th stop of the slice is row
+      // first_row + s (reading P6), so this thread's stops take the rows from
+      // first_row + tile_rank + nx on; the tile's first segment waits for its carry-in
+      // (below), every other segment is complete
+      const int f0 = __ffs(stops) - 1;
+      const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
+      const int row_first = frk + trank + nx;
+      VT fpr = VT(0);  // the first segment's own part (registers: no dynamic indexing)
 #pragma unroll
-          for (int i = 0; i < BT; ++i) {
-            const int b = bt0 + i;
-            if (b < tb1) {
-              if (b >= sh.sp[k + 1]) k = slice_of(b, k);
-              if (k == kk) {
-                run = run + pr[i];
-                if ((stops >> i) & 1u) {
-                  const VT val = first ? run + Vex : run;
-                  first = false;
-                  const bool res = k < k_lo + PANEL_NBUF;
-                  const int64_t rec = (p * KS + k) * (int64_t)NW;
-                  const uint32_t* oc = res ? occ_of(k) : a.occ + rec;
-                  row = row < 0 ? select_row(oc, res ? pre_of(k) : a.pre + rec, NW, s - sh.st[k]) : next_row(oc, row);
-                  acc[row] = acc[row] + val;
-                  ++s;
-                  run = VT(0);
-                }
-              }
-            }
+      for (int i = 0; i < BT; ++i)  // the first stop: + earlier lanes now, or deferred (dep)
+        if (i == f0) {
+          fpr = pr[i];
+          pr[i] = dep ? VT(0) : pr[i] + vx;
+        }
+      {
+        VT* ar = acc + row_first;
+#pragma unroll
+        for (int i = 0; i < BT; ++i)
+          if ((stops >> i) & 1u) {
+            *ar = *ar + pr[i];
+            ++ar;
+          }
+      }
+      // ---- carry-in of the first segment: decoupled look-back over the slice's earlier
+      // tiles (fold newest first back to the nearest tile holding a row stop)
+      const unsigned dball = __ballot_sync(0xffffffffu, dep);
+      if (dball) {
+        VT carry = VT(0);
+        if (lane == 0) {
+          for (int q = lt - 1; q >= ltile_k; --q) {
+            while (sh.rtag[q % RING] != q + 1) __nanosleep(16);
+            __threadfence_block();
+            carry = sh.rT[q % RING] + carry;
+            if (sh.rH[q % RING]) break;
           }
         }
-        __syncthreads();
+        carry = __shfl_sync(0xffffffffu, carry, 0);
+        if (dep) acc[row_first] = acc[row_first] + (fpr + (vx + carry));
       }
     }
-    if (t == 0) {
-      sh.cin = Fall ? Vall : cin + Vall;  // the tile's open segment carries into the next tile
-      sh.s_before = sb + Ntot;
-    }
+    // ---- slice done: every row has its slice-k sum before any slice-(k+1) sum --------
     __syncthreads();
+    const int k2 = next_nonempty(k + 1);
+    if (t == 0 && k2 < KS) {
+      const int k3 = next_nonempty(k2 + 1);
+      if (k3 < KS) issue(k3, o + 2);  // into the buffer of slice k, finished
+    }
+    k = k2;
+    ++o;
   }
 
   // ---- epilogue: y := acc (scaled), sum of y^2 ----------------------------------------
   const double inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
-  for (int r = t; r < rows; r += BC) {
-    const VT o = (a.epi & 1) ? (VT)(acc[r] * inv) : acc[r];
-    y[row0 + r] = o;
-    ssq += (double)o * (double)o;
+  for (int r = t; r < rows; r += NTH) {
+    const VT o2 = (a.epi & 1) ? (VT)(acc[r] * inv) : acc[r];
+    y[row0 + r] = o2;
+    ssq += (double)o2 * (double)o2;
   }
   if (a.epi & 2) {
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) ssq += __shfl_xor_sync(0xffffffffu, ssq, o);
+    for (int d = 16; d > 0; d >>= 1) ssq += __shfl_xor_sync(0xffffffffu, ssq, d);
     if (lane == 0) sh.ss[wid] = ssq;
     __syncthreads();
     if (t == 0) {
@@ -400,14 +365,17 @@ int panel_attr(int64_t R, int64_t W, int* regs) {
   cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   const size_t need = panel_smem_bytes(R, W);
   if (need + fa.sharedSizeBytes > (size_t)optin) return (int)cudaErrorInvalidConfiguration;
-  return (int)cudaFuncSetAttribute(panel_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   optin - (int)fa.sharedSizeBytes);
+  e = cudaFuncSetAttribute(panel_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           optin - (int)fa.sharedSizeBytes);
+  if (e != cudaSuccess) return (int)e;
+  // two CTAs per SM when the windows allow it: the whole unified carve-out as shared memory
+  return (int)cudaFuncSetAttribute(panel_kernel<float>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
 }
 
 int launch_panel(const PanelArgs& a, int dtype, void* stream) {
   if (dtype != 0) return (int)cudaErrorNotSupported;
   if (a.npanels == 0) return 0;
-  panel_kernel<float><<<(unsigned)a.npanels, BC, panel_smem_bytes(a.R, a.W), (cudaStream_t)stream>>>(a);
+  panel_kernel<float><<<(unsigned)a.npanels, NTH, panel_smem_bytes(a.R, a.W), (cudaStream_t)stream>>>(a);
   return (int)cudaGetLastError();
 }
 

@@ -159,10 +159,22 @@ class Matrix:
     def launches_per_spmv(self) -> int:
         return int(lib.yaspmv_launches_per_spmv(self._h))
 
+    def profile_begin(self) -> None:
+        """Record CUDA events around every kernel group of the following SpMVs."""
+        check(lib.yaspmv_profile_begin(self._h))
+
+    def profile_end(self) -> dict:
+        """Summed device milliseconds per stage since profile_begin(): plain/far part,
+        band kernel, band y^2 sum; and the number of calls."""
+        ms = (ctypes.c_double * 3)()
+        calls = ctypes.c_int64()
+        check(lib.yaspmv_profile_end(self._h, ms, 3, ctypes.byref(calls)))
+        return {"plain_ms": ms[0], "band_ms": ms[1], "band_sum_ms": ms[2], "calls": calls.value}
+
     _ARR_DT = {"flags": np.uint8, "col_delta": np.int16, "seg_row": np.int32, "zero_rows": np.int32,
                "cta_seg0": np.int32, "fre": np.int32, "band_flags": np.uint8, "band_col16": np.uint16,
                "band_panel_blk0": np.int64, "band_slice_ptr": np.int32, "band_stop_ptr": np.int32,
-               "band_occ": np.uint32, "band_pre": np.uint16}
+               "band_first_row": np.int32, "band_tile_rank": np.int32}
 
     def _arr_dtype(self, name: str):
         if name.startswith("val") or name == "band_val":

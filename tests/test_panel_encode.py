@@ -28,8 +28,8 @@ def _compare(csr, R, W, B, col0=0, far=(16, 256, 0, 0)):
         assert np.array_equal(A.export("band_panel_blk0"), enc.panel_blk0)
         assert np.array_equal(A.export("band_slice_ptr"), enc.slice_ptr.ravel())
         assert np.array_equal(A.export("band_stop_ptr"), enc.stop_ptr.ravel())
-        assert np.array_equal(A.export("band_occ"), enc.occ.ravel())
-        assert np.array_equal(A.export("band_pre"), enc.pre.ravel())
+        assert np.array_equal(A.export("band_first_row"), enc.first_row.ravel())
+        assert np.array_equal(A.export("band_tile_rank"), enc.tile_rank)
         f = enc.far
         assert (info["nnzb"], info["nnzb_pad"], info["ntiles"], info["n_stops"]) == \
             (f.nnzb, f.nnzb_pad, f.ntiles, f.n_stops)

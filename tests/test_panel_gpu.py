@@ -59,6 +59,11 @@ CASES = {
     "all-band": (lambda: synth.circuit_like_rows(0, 9_000, n=9_000, band=500, n_net=0, p_local=1.0),
                  dict(B=20000, R=8192, W=4096)),
     "tiny-m": (lambda: synth.random_tiny(3, dtype=np.float32, m=17, n=23), dict(B=8, R=256, W=8)),
+    # far part as BCCOO+ (S = 2): its slice results are combined by the band kernel
+    "c5-scaled-far-S2": (lambda: synth.circuit_like_rows(0, 400_000, n=400_000, band=8192, n_net=4,
+                                                         net_log2=(12, 16)),
+                         dict(B=8192, R=4096, W=1024, S=2, T=32, C=128, col_mode=E.COL_I32)),
+    "webbase-far-S3": (lambda: synth.webbase_like(m=200_000), dict(B=1024, R=4096, W=512, S=3)),
 }
 
 
@@ -80,7 +85,7 @@ def test_tolerance_and_determinism(name):
         A.free()
 
 
-@pytest.mark.parametrize("name", ["c5-scaled", "small-many-slices", "col0-neg", "tiny-m"])
+@pytest.mark.parametrize("name", ["c5-scaled", "small-many-slices", "col0-neg", "tiny-m", "c5-scaled-far-S2"])
 def test_integer_exact(name):
     mk, params = CASES[name]
     csr0 = mk()
@@ -103,7 +108,7 @@ def test_device_arrays_equal_oracle(name):
     from paper_conf_ppopp_yanlzz14_b200._lib import PANEL_BC, PANEL_BT
     far = E.Params(1, 1, 1, params.get("T", 16), params.get("C", 256), params.get("col_mode", 0),
                    params.get("empty_mode", 0))
-    pp = PN.PanelParams(R=params.get("R", 16384), W=params.get("W", 8192), B=params["B"], T=PANEL_BT, C=PANEL_BC,
+    pp = PN.PanelParams(R=params.get("R", 16384), W=params.get("W", 16384), B=params["B"], T=PANEL_BT, C=PANEL_BC,
                         diag0=params.get("col0", 0), far=far)
     enc = PN.encode_panel(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, pp)
     A = _build(csr, **params)
@@ -111,8 +116,8 @@ def test_device_arrays_equal_oracle(name):
         assert np.array_equal(A.export("band_flags", device=True), enc.flags)
         assert np.array_equal(A.export("band_col16", device=True), enc.col16)
         assert np.array_equal(A.export("band_val", device=True).view(np.uint32), enc.val.view(np.uint32))
-        assert np.array_equal(A.export("band_occ", device=True), enc.occ.ravel())
-        assert np.array_equal(A.export("band_pre", device=True), enc.pre.ravel())
+        assert np.array_equal(A.export("band_first_row", device=True), enc.first_row.ravel())
+        assert np.array_equal(A.export("band_tile_rank", device=True), enc.tile_rank)
         assert np.array_equal(A.export("band_slice_ptr", device=True), enc.slice_ptr.ravel())
         assert np.array_equal(A.export("band_stop_ptr", device=True), enc.stop_ptr.ravel())
         assert np.array_equal(A.export("flags", device=True), enc.far.flags)
@@ -133,7 +138,7 @@ def test_gpu_encoded_far_part():
         A.free()
 
 
-@pytest.mark.parametrize("name", ["c5-scaled", "webbase"])
+@pytest.mark.parametrize("name", ["c5-scaled", "webbase", "webbase-far-S3"])
 def test_power_step(name):
     mk, params = CASES[name]
     csr0 = mk()
