@@ -298,9 +298,10 @@ def main():
                     "check with several ranks on one GPU; never a performance number)")
     ap.add_argument("--rows", type=int, default=0, help="C5 only: use the first ROWS rows/cols (checks)")
     ap.add_argument("--exchange", default="auto", choices=["auto", "fused", "nccl"],
-                    help="x replication for N > 1: fused = SpMV write-back into every rank's x over peer "
-                         "memory (yaspmv_power_step_fused, CUDA IPC); nccl = all_reduce + all_gather_into_tensor. "
-                         "auto: fused for N > 1 (nccl if IPC mapping fails), none for N = 1")
+                    help="x replication for N > 1: nccl = all_reduce + all_gather_into_tensor (the default "
+                         "until the fused path has run across devices); fused = SpMV write-back into every "
+                         "rank's x over peer memory (yaspmv_power_step_fused, CUDA IPC, plain BCCOO/BCCOO+ "
+                         "only). auto: nccl for N > 1 (the fused step is timed as extra keys when it can run)")
     args = ap.parse_args()
 
     world = _env_int("WORLD_SIZE", 1)
@@ -332,6 +333,8 @@ def main():
     params = dict(DEFAULT_PARAMS.get(args.config, {}))
     if args.params:
         params.update(json.loads(args.params))
+    if params.get("B", 0) and world > 1:
+        params["col0"] = L.rank * L.m_max  # the rank's diagonal in the padded column space
     big = csr.nnz > 50_000_000
     # DROP_CSR (no host copy kept) + GPU translation to BCCOO for the 1B-nnz matrix
     params.setdefault("flags", (2 | 4) if big else 0)
@@ -345,7 +348,7 @@ def main():
     stream = torch.cuda.current_stream()
     exchange = args.exchange
     if exchange == "auto":
-        exchange = "fused" if world > 1 else "none"
+        exchange = "nccl" if world > 1 else "none"
     fpit = None
     if exchange == "fused":
         try:
@@ -454,6 +457,36 @@ def main():
            "api": "yaspmv_spmv_host_async + yaspmv_host_sync (pinned x in, y out every step, per rank)",
            "steps": args.e2e_steps}
 
+    # ---- N > 1: the fused exchange (peer stores from the SpMV epilogue) as extra keys ---
+    fused_info = None
+    if world > 1 and fpit is None and args.exchange == "auto":
+        if info["band_blocks_pad"] > 0:
+            fused_info = {"unavailable": "panel-sliced BCCOO+ handle: the fused exchange runs the plain format only"}
+        else:
+            try:
+                fp = D.FusedPowerIteration(L, A, tdt, dev, timeout_ms=20000)
+                for _ in range(3):
+                    fp.step(stream)
+                fp.comm.wait(stream)
+                torch.cuda.synchronize()
+                dist.barrier()
+                f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                f0.record(stream)
+                for _ in range(20):
+                    fp.step(stream)
+                fp.comm.wait(stream)
+                f1.record(stream)
+                torch.cuda.synchronize()
+                fp.comm.check()
+                tf = torch.tensor([f0.elapsed_time(f1) / 20], dtype=torch.float64, device=dev)
+                dist.all_reduce(tf, op=dist.ReduceOp.MAX)
+                fused_info = {"ms_per_step": float(tf.item()), "steps": 20,
+                              "gflops": 2.0 * nnz_total / (float(tf.item()) * 1e-3) / 1e9}
+                dist.barrier()
+                fp.comm.free()
+            except Exception as e:  # never fail the bench line on the optional path
+                fused_info = {"error": f"{type(e).__name__}: {e}"[:300]}
+
     if rank == 0:
         peak, peak_kind = measured_peaks()
         achieved = info["alg_bytes"] / (spmv_ms * 1e-3) / 1e9
@@ -511,7 +544,7 @@ def main():
                                           for k, v in kern.items()}},
             "gpu_launches": (fpit.launches_per_step() if fpit is not None else A.launches_per_power_step())
                             * args.steps,
-            "clocks": clocks, "e2e": e2e,
+            "clocks": clocks, "e2e": e2e, "fused_exchange": fused_info,
             "build": {"generate_s": t_gen, "build_s": t_build, "encode_upload_s": info["build_seconds"]},
         }
         if world == 1 and not args.no_cpu_baseline:

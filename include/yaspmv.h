@@ -263,6 +263,12 @@ enum {
 yaspmv_status yaspmv_export(yaspmv_matrix A, int32_t which, void* host_dst, int64_t bytes, int64_t* nbytes);
 yaspmv_status yaspmv_export_device(yaspmv_matrix A, int32_t which, void* host_dst, int64_t bytes,
                                    int64_t* nbytes);
+/* yaspmv_export_device_range: as yaspmv_export_device for the workgroup tiles
+ * [first_tile, first_tile + ntiles) only (per-block arrays: the tiles' T*C blocks — 512 for the
+ * band stream; CTA_SEG0 / BAND_TILE_RANK: those tiles' entries), for checking windows of
+ * matrices whose full arrays are too large to copy. */
+yaspmv_status yaspmv_export_device_range(yaspmv_matrix A, int32_t which, int64_t first_tile, int64_t ntiles,
+                                         void* host_dst, int64_t bytes, int64_t* nbytes);
 
 /* ---------------------------------------------------------------- power-iteration helpers
  * yaspmv_nrm2sq: out_dev[0] (device double) := sum_i v[i]^2 over device v[n] of `dtype`,

@@ -31,7 +31,7 @@ IPC_HANDLE_BYTES = 64
 # every symbol include/yaspmv.h declares (checked by tests/test_abi.py)
 EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv", "yaspmv_spmv_host",
             "yaspmv_tune", "yaspmv_reencode", "yaspmv_get_info", "yaspmv_export", "yaspmv_export_device",
-            "yaspmv_nrm2sq", "yaspmv_nrm2sq_scratch_bytes", "yaspmv_scale", "yaspmv_last_error",
+            "yaspmv_nrm2sq", "yaspmv_nrm2sq_scratch_bytes", "yaspmv_export_device_range", "yaspmv_scale", "yaspmv_last_error",
             "yaspmv_version", "yaspmv_launches_per_spmv", "yaspmv_spmv_host_async", "yaspmv_host_sync",
             "yaspmv_spmv_power", "yaspmv_launches_per_power_step", "yaspmv_tune_ex",
             "yaspmv_comm_create", "yaspmv_comm_ipc_handle", "yaspmv_comm_open_ipc", "yaspmv_comm_connect_local",
@@ -105,6 +105,7 @@ def _load():
         "yaspmv_get_info": ([H, ctypes.POINTER(Info)], ctypes.c_int),
         "yaspmv_export": ([H, i32, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),
         "yaspmv_export_device": ([H, i32, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),
+        "yaspmv_export_device_range": ([H, i32, i64, i64, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),
         "yaspmv_nrm2sq": ([vp, i64, ctypes.c_int, vp, vp, vp], ctypes.c_int),
         "yaspmv_nrm2sq_scratch_bytes": ([i64], i64),
         "yaspmv_scale": ([vp, vp, i64, ctypes.c_int, vp, vp], ctypes.c_int),

@@ -202,6 +202,53 @@ yaspmv_status yaspmv_export_device(yaspmv_matrix A, int32_t which, void* dst, in
   return YASPMV_OK;
 }
 
+yaspmv_status yaspmv_export_device_range(yaspmv_matrix A, int32_t which, int64_t first_tile, int64_t ntiles,
+                                         void* dst, int64_t bytes, int64_t* nbytes) {
+  if (!A) return fail(YASPMV_EINVAL, "NULL handle");
+  if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle has no device arrays");
+  ArrDesc d;
+  yaspmv_status st = describe(A, which, d);
+  if (st != YASPMV_OK) return st;
+  const Canonical& c = A->can;
+  // bytes of one workgroup tile of the array (per-tile arrays: one entry)
+  int64_t tb = 0, total_tiles = 0;
+  const bool band = which >= YASPMV_ARR_BAND_FLAGS;
+  const int64_t TC = band ? PANEL_TC : (int64_t)c.p.T * c.p.C;
+  const int64_t ntl = band ? A->pan.nband_pad / PANEL_TC : c.ntiles;
+  switch (which) {
+    case YASPMV_ARR_FLAGS:
+    case YASPMV_ARR_BAND_FLAGS: tb = TC / 8; break;
+    case YASPMV_ARR_CTA_SEG0:
+    case YASPMV_ARR_BAND_TILE_RANK: tb = 4; break;
+    case YASPMV_ARR_COL:
+    case YASPMV_ARR_COL_DELTA:
+    case YASPMV_ARR_VAL0:
+    case YASPMV_ARR_VAL1:
+    case YASPMV_ARR_VAL2:
+    case YASPMV_ARR_VAL3:
+    case YASPMV_ARR_BAND_COL16:
+    case YASPMV_ARR_BAND_VAL: tb = ntl > 0 ? d.bytes / ntl : 0; break;
+    default: return fail(YASPMV_EINVAL, "range export: per-block or per-tile arrays only");
+  }
+  total_tiles = ntl;
+  if (first_tile < 0 || ntiles < 0 || first_tile + ntiles > total_tiles) return fail(YASPMV_EINVAL, "tile range out of bounds");
+  const int64_t out = ntiles * tb;
+  if (nbytes) *nbytes = out;
+  if (!dst || out == 0) return YASPMV_OK;
+  if (bytes < out) return fail(YASPMV_EINVAL, "destination too small");
+  CUDA_TRY(cudaSetDevice(A->device));
+  CUDA_TRY(cudaDeviceSynchronize());
+  const uint8_t* src = static_cast<const uint8_t*>(d.dev) + first_tile * tb;
+  if (d.ptb == 0) {
+    CUDA_TRY(cudaMemcpy(dst, src, out, cudaMemcpyDeviceToHost));
+  } else {
+    std::vector<uint8_t> tmp(out);
+    CUDA_TRY(cudaMemcpy(tmp.data(), src, out, cudaMemcpyDeviceToHost));
+    permute_from_device_layout(tmp.data(), static_cast<uint8_t*>(dst), ntiles, d.ntiles >= 0 ? d.C : c.p.C, d.ptb);
+  }
+  return YASPMV_OK;
+}
+
 // ------------------------------------------------------------------ auto-tuner (§4)
 yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode) {
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");

@@ -105,6 +105,40 @@ struct PanelShared {
   double ss[NWARP];
 };
 
+// Thread 0 requests the x window of the o-th non-empty slice of the panel (its slice id
+// found from the slice offsets) into buffer o % NBUF: W values of x from column cb + k*W
+// with cp.async.bulk on the buffer's mbarrier, the unaligned ends by plain loads, and the
+// zero slot behind the window (the column of a FILLER block, reading P6).
+template <typename VT>
+__device__ __forceinline__ void issue_window(PanelShared& sh, unsigned char* bufs, int64_t bufbytes, const VT* x,
+                                          int64_t n, int64_t xe, int64_t cb, int W, int KS, int o) {
+  int k = 0, oo = -1;
+  for (; k < KS; ++k)
+    if (sh.sp[k] != sh.sp[k + 1] && ++oo == o) break;
+  if (k >= KS) return;
+  uint64_t* bar = &sh.bar[o % PANEL_NBUF];
+  if (o >= PANEL_NBUF) mbar_wait(bar, (unsigned)((o / PANEL_NBUF - 1) & 1));  // previous use landed
+  VT* w = reinterpret_cast<VT*>(bufs + (o % PANEL_NBUF) * bufbytes);
+  const int64_t base = cb + (int64_t)k * W;
+  const int sh_k = (int)(((xe + base) % 4 + 4) % 4);
+  const int64_t lo = max((int64_t)0, base), hi = min(n, base + W);
+  unsigned tx = 0;
+  int64_t alo = lo, ahi = lo;
+  if (lo < hi) {
+    alo = lo + ((4 - ((xe + lo) & 3)) & 3);
+    ahi = hi - ((xe + hi) & 3);
+    if (alo > ahi) alo = ahi = hi;
+    for (int64_t j = lo; j < alo && j < hi; ++j) w[sh_k + (j - base)] = x[j];  // unaligned head
+    for (int64_t j = max(ahi, alo); j < hi; ++j) w[sh_k + (j - base)] = x[j];  // unaligned tail
+    tx += (unsigned)((ahi - alo) * sizeof(VT));
+  }
+  w[sh_k + W] = VT(0);
+  mbar_arrive_tx(bar, tx);
+  if (ahi > alo) bulk_g2s(w + sh_k + (alo - base), x + alo, (unsigned)((ahi - alo) * sizeof(VT)), bar);
+  __threadfence_block();
+  sh.armed[o % PANEL_NBUF] = o;
+}
+
 template <typename VT>
 __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   extern __shared__ __align__(16) unsigned char dsm[];
@@ -166,31 +200,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     while (k < KS && sh.sp[k] == sh.sp[k + 1]) ++k;
     return k;
   };
-  // thread 0 requests the window of slice k (non-empty ordinal o) into buffer o % NBUF
-  // (FILLER blocks read the zero slot behind the window)
-  auto issue = [&](int k, int o) {
-    uint64_t* bar = &sh.bar[o % PANEL_NBUF];
-    if (o >= PANEL_NBUF) mbar_wait(bar, (unsigned)((o / PANEL_NBUF - 1) & 1));  // previous use landed
-    VT* w = win(o);
-    const int sh_k = shift_of(k);
-    const int64_t base = cb + (int64_t)k * W;
-    const int64_t lo = max((int64_t)0, base), hi = min((int64_t)a.n, base + W);
-    unsigned tx = 0;
-    int64_t alo = lo, ahi = lo;
-    if (lo < hi) {
-      alo = lo + ((4 - ((xe + lo) & 3)) & 3);
-      ahi = hi - ((xe + hi) & 3);
-      if (alo > ahi) alo = ahi = hi;
-      for (int64_t j = lo; j < alo && j < hi; ++j) w[sh_k + (j - base)] = x[j];  // unaligned head
-      for (int64_t j = max(ahi, alo); j < hi; ++j) w[sh_k + (j - base)] = x[j];  // unaligned tail
-      tx += (unsigned)((ahi - alo) * sizeof(VT));
-    }
-    w[sh_k + W] = VT(0);
-    mbar_arrive_tx(bar, tx);
-    if (ahi > alo) bulk_g2s(w + sh_k + (alo - base), x + alo, (unsigned)((ahi - alo) * sizeof(VT)), bar);
-    __threadfence_block();
-    sh.armed[o % PANEL_NBUF] = o;
-  };
+  auto issue = [&](int o) { issue_window<VT>(sh, bufs, L.bufbytes, x, a.n, xe, cb, W, KS, o); };
 
   const int64_t pb0 = a.panel_blk0[p];
   const int64_t tile0 = pb0 / PANEL_TC;  // first tile of the panel
@@ -202,14 +212,48 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   // this warp's tiles: in each non-empty slice, the slice's tiles wid, wid + NWARP, ...
   int k = next_nonempty(0);
   int o = 0;  // non-empty ordinal of slice k
-  if (t == 0 && k < KS) {
-    issue(k, 0);
-    const int k1 = next_nonempty(k + 1);
-    if (k1 < KS) issue(k1, 1);
-  }
+
   double ssq = 0.0;
 
+  // Warp NWARP-1 is the window producer; warps 0..NWARP-2 compute.  Between slices every
+  // acc[row] must receive its slice o-1 sum before its slice o sum, and slice o-1's window
+  // buffer may take slice o+1 only when no warp reads it any more: named barrier X_o
+  // (bar.sync 1 + (o & 1), all NTH threads).  A compute warp that is done with slice o-1
+  // loads, multiplies and scans its first slice-o tile, and waits on X_o only before that
+  // tile's first acc update; the producer passes X_o and requests window o+1.
+  constexpr int NCW = NWARP - 1;
+  if (wid == NWARP - 1) {
+    int nne = 0;
+    for (int kk = 0; kk < KS; ++kk) nne += sh.sp[kk] != sh.sp[kk + 1];
+    if (lane == 0) {
+      issue(0);
+      issue(1);
+    }
+    for (int oo = 1; oo < nne; ++oo) {
+      if (oo & 1) asm volatile("bar.sync 2, %0;" ::"n"(NTH) : "memory");
+      else asm volatile("bar.sync 1, %0;" ::"n"(NTH) : "memory");
+      if (lane == 0) issue(oo + 1);
+    }
+    k = KS;  // no tiles for the producer
+  }
+  auto slice_barrier = [&](int oo) {
+    if (oo & 1) asm volatile("bar.sync 2, %0;" ::"n"(NTH) : "memory");
+    else asm volatile("bar.sync 1, %0;" ::"n"(NTH) : "memory");
+  };
+  uint32_t vw[VCH * 4], cw[CCH * 4], fl = 0;
+  int trank = 0;
+  auto load_tile = [&](int lt) {  // panel-local tile: the thread's run (device layout)
+    const int64_t tile = tile0 + lt;
+#pragma unroll
+    for (int c = 0; c < CCH; ++c) ld16(cbase + (tile * (int64_t)32 * CCH + (int64_t)c * 32 + lane) * 16, pol, &cw[4 * c]);
+#pragma unroll
+    for (int c = 0; c < VCH; ++c) ld16(vbase + (tile * (int64_t)32 * VCH + (int64_t)c * 32 + lane) * 16, pol, &vw[4 * c]);
+    fl = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
+    trank = __ldg(a.tile_rank + tile);
+  };
   while (k < KS) {
+    const int ltile_k = sh.sp[k] >> 9;                     // panel-local first tile of the slice
+    const int ntile_k = (sh.sp[k + 1] - sh.sp[k]) >> 9;    // tiles of the slice
     // window o of slice k resident (a buffer two requests behind would alias the awaited
     // parity: wait until the request is armed first)
     while (sh.armed[o % PANEL_NBUF] != o) {
@@ -217,23 +261,17 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     mbar_wait(&sh.bar[o % PANEL_NBUF], (o / PANEL_NBUF) & 1);
     const VT* wk = win(o) + shift_of(k);
     const int frk = sh.fr[k];
-    const int ltile_k = sh.sp[k] >> 9;                     // panel-local first tile of the slice
-    const int ntile_k = (sh.sp[k + 1] - sh.sp[k]) >> 9;    // tiles of the slice
-    for (int u = wid; u < ntile_k; u += NWARP) {
+    bool pending = o > 0;  // X_o still ahead of this warp
+    for (int u = wid; u < ntile_k; u += NCW) {
       const int lt = ltile_k + u;       // panel-local tile index (tag of its carry record)
-      const int64_t tile = tile0 + lt;  // global tile index
-      // ---- stream the thread tile: 128-bit loads of the device layout -----
-      uint32_t vw[VCH * 4], cw[CCH * 4];
-#pragma unroll
-      for (int c = 0; c < CCH; ++c) ld16(cbase + (tile * (int64_t)32 * CCH + (int64_t)c * 32 + lane) * 16, pol, &cw[4 * c]);
-#pragma unroll
-      for (int c = 0; c < VCH; ++c) ld16(vbase + (tile * (int64_t)32 * VCH + (int64_t)c * 32 + lane) * 16, pol, &vw[4 * c]);
-      const uint32_t fl = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
-      const int trank = __ldg(a.tile_rank + tile);
-      // flow control: the record slot of this tile must have been released
-      if (lt >= LAG && lane == 0)
-        while (sh.rtag[(lt - LAG) % RING] != lt - LAG + 1) __nanosleep(32);
-      __syncwarp();
+      load_tile(lt);
+      // flow control (slices of more than LAG tiles only): the record slot of this tile
+      // must have been released
+      if (ntile_k > LAG && u >= LAG) {
+        if (lane == 0)
+          while (sh.rtag[(lt - LAG) % RING] != lt - LAG + 1) __nanosleep(32);
+        __syncwarp();
+      }
 
       // ---- multiply: gathers from the slice's window --------------------------------
       VT pr[BT];
@@ -277,26 +315,25 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
         nx = 0;
         vx = VT(0);
       }
+      if (pending) {  // every warp is done with slice o - 1 (acc order)
+        slice_barrier(o);
+        pending = false;
+      }
       // ---- add the segment sums to acc[row]: the s-th stop of the slice is row
       // first_row + s (reading P6), so this thread's stops take the rows from
-      // first_row + tile_rank + nx on; the tile's first segment waits for its carry-in
-      // (below), every other segment is complete
-      const int f0 = __ffs(stops) - 1;
+      // first_row + tile_rank + nx on.  The first stop also gets the earlier lanes' part
+      // (vx); when it continues earlier tiles (dep) their carry is added below, after the
+      // look-back — a fixed association, so y stays bitwise deterministic
       const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
       const int row_first = frk + trank + nx;
-      VT fpr = VT(0);  // the first segment's own part (registers: no dynamic indexing)
-#pragma unroll
-      for (int i = 0; i < BT; ++i)  // the first stop: + earlier lanes now, or deferred (dep)
-        if (i == f0) {
-          fpr = pr[i];
-          pr[i] = dep ? VT(0) : pr[i] + vx;
-        }
       {
         VT* ar = acc + row_first;
+        VT add = vx;
 #pragma unroll
         for (int i = 0; i < BT; ++i)
           if ((stops >> i) & 1u) {
-            *ar = *ar + pr[i];
+            *ar = *ar + (pr[i] + add);
+            add = VT(0);
             ++ar;
           }
       }
@@ -314,19 +351,14 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
           }
         }
         carry = __shfl_sync(0xffffffffu, carry, 0);
-        if (dep) acc[row_first] = acc[row_first] + (fpr + (vx + carry));
+        if (dep) acc[row_first] = acc[row_first] + carry;
       }
     }
-    // ---- slice done: every row has its slice-k sum before any slice-(k+1) sum --------
-    __syncthreads();
-    const int k2 = next_nonempty(k + 1);
-    if (t == 0 && k2 < KS) {
-      const int k3 = next_nonempty(k2 + 1);
-      if (k3 < KS) issue(k3, o + 2);  // into the buffer of slice k, finished
-    }
-    k = k2;
+    if (pending) slice_barrier(o);  // no tile of this slice: still part of X_o
+    k = next_nonempty(k + 1);
     ++o;
   }
+  __syncthreads();  // the last slice's sums are in acc
 
   // ---- epilogue: y := acc (scaled), sum of y^2 ----------------------------------------
   const double inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;

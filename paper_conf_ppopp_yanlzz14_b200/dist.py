@@ -202,8 +202,20 @@ class FusedPowerIteration:
             if layout.world > 1:
                 import torch.distributed as dist
                 self._agree(err, group, "create the exchange buffers")
+                # the IPC handle too is agreed on: a rank that cannot export its buffer
+                # gathers None instead of raising before the collective (no rank hangs)
+                try:
+                    mine = comm.ipc_handle()
+                except Exception as e:
+                    mine, err = None, e
                 handles = [None] * layout.world
-                dist.all_gather_object(handles, comm.ipc_handle(), group=group)
+                dist.all_gather_object(handles, mine, group=group)
+                try:
+                    self._agree(err, group, "export the IPC handles")
+                except RuntimeError:
+                    if hasattr(comm, "free"):
+                        comm.free()
+                    raise
                 try:
                     comm.open_ipc(handles)
                 except Exception as e:
@@ -232,9 +244,18 @@ class FusedPowerIteration:
 
     def restart(self):
         """x_0 = 1/sqrt(N) on the real entries of this rank's copy, then (world > 1, own comm)
-        a barrier so that no peer writes into a buffer before every rank is ready."""
+        a barrier so that no peer writes into a buffer before every rank is ready.  Before
+        x_0 is written, every peer's last step must be over: its SpMV stores z rows into this
+        rank's buffers over peer memory (wait for the peers on the device, synchronize,
+        barrier)."""
         import torch
         L = self.L
+        if self.own_comm and L.world > 1 and getattr(self, "first", None) is False:
+            import torch.distributed as dist
+            self.comm.wait(None)
+            if self.device.type == "cuda":
+                torch.cuda.synchronize(self.device)
+            dist.barrier(group=self.group)
         x = self.comm.x(0)
         x.zero_()
         n_true = int(L.bounds[-1])

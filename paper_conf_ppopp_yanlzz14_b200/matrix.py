@@ -193,6 +193,16 @@ class Matrix:
         check(fn(self._h, _lib.ARR[name], out.ctypes.data if nb.value else None, nb.value, ctypes.byref(nb)))
         return out.view(self._arr_dtype(name))
 
+    def export_range(self, name: str, first_tile: int, ntiles: int) -> np.ndarray:
+        """Canonical array `name` for workgroup tiles [first_tile, first_tile + ntiles),
+        read back from the device (yaspmv_export_device_range)."""
+        nb = ctypes.c_int64()
+        check(lib.yaspmv_export_device_range(self._h, _lib.ARR[name], first_tile, ntiles, None, 0, ctypes.byref(nb)))
+        out = np.empty(nb.value, dtype=np.uint8)
+        check(lib.yaspmv_export_device_range(self._h, _lib.ARR[name], first_tile, ntiles,
+                                              out.ctypes.data if nb.value else None, nb.value, ctypes.byref(nb)))
+        return out.view(self._arr_dtype(name))
+
 
 class Comm:
     """The replicated x of a row-partitioned power iteration (yaspmv_comm, include/yaspmv.h

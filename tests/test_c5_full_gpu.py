@@ -65,3 +65,69 @@ def test_c5_power_step_sampled_rows(c5):
     assert ok, worst
     yy = y.cpu().numpy().astype(np.float64)
     assert abs(out.item() - float(np.dot(yy, yy))) <= 1e-6 * out.item()
+
+
+def _panel_windows(csr, R):
+    """Panel windows to check: the first two panels, the panel of the longest net row,
+    the last two panels."""
+    from synth import matrices as sm
+    net, ln = sm.c5_net_rows()
+    npan = -(-csr.m // R)
+    pn = int(net[np.argmax(ln)]) // R
+    return sorted({(0, 2), (pn, pn + 1), (npan - 2, npan)})
+
+
+def test_c5_encoding_windows_bit_exact(c5):
+    """north_star "Encoded arrays and row-segment boundaries must match bit-exactly" at C5
+    scale: windows of the device arrays of the bench's handle (host panel encoder for the
+    band stream, GPU translation, for the BCCOO+ far part) against oracle/encode.py
+    and oracle/panel.py run on the same rows (P:114, P:119, P:121, P:148-153, P:188-189;
+    readings P1-P6)."""
+    from oracle import encode as E, panel as PN
+    csr, A = c5
+    info = A.info()
+    prm = info["params"]
+    R, W, B = prm["panel_rows"], prm["slice_width"], prm["band"]
+    S, T, C = prm["slices"], prm["thread_tile"], prm["cta_size"]
+    assert B > 0 and info["band_panels"] == -(-csr.m // R)
+    blk0 = A.export("band_panel_blk0", device=True)
+    sptr = A.export("band_slice_ptr", device=True).reshape(info["band_panels"], -1)
+    frow = A.export("band_first_row", device=True).reshape(info["band_panels"], -1)
+    far_flags = np.unpackbits(A.export("flags", device=True), bitorder="little")
+    far_stop = np.flatnonzero(far_flags[: info["nnzb"]] == 0)      # FILLER: stop k ends stacked row k
+    assert prm["empty_mode"] == E.EMPTY_FILLER and far_stop.size == S * csr.m
+    TCf = T * C
+    for p0, p1 in _panel_windows(csr, R):
+        r0, r1 = p0 * R, min(csr.m, p1 * R)
+        sub = csr.row_slice(r0, r1)
+        pp = PN.PanelParams(R=R, W=W, B=B, T=16, C=32, diag0=r0,
+                            far=E.Params(1, 1, S, T, C, prm["col_mode"], E.EMPTY_FILLER))
+        # the window's slices use the full matrix' slice width of the far part
+        enc = PN.encode_panel(sub.m, csr.n, sub.row_ptr, sub.col, sub.val, pp)
+        # band stream: panels are independent, so the window's arrays are a slice of the whole
+        assert np.array_equal(sptr[p0:p1], enc.slice_ptr) and np.array_equal(frow[p0:p1], enc.first_row)
+        t0, nt = int(blk0[p0]) // 512, (int(blk0[p1]) - int(blk0[p0])) // 512
+        assert nt == enc.nband_pad // 512
+        assert np.array_equal(A.export_range("band_flags", t0, nt), enc.flags)
+        assert np.array_equal(A.export_range("band_col16", t0, nt), enc.col16)
+        assert np.array_equal(A.export_range("band_val", t0, nt).view(np.uint32), enc.val.view(np.uint32))
+        assert np.array_equal(A.export_range("band_tile_rank", t0, nt), enc.tile_rank)
+        # far part (BCCOO+, S slices stacked top-down, P:148-153): stacked rows s*m + [r0, r1)
+        ef = enc.far
+        ebits = np.unpackbits(ef.flags, bitorder="little")[: ef.nnzb]
+        estop = np.flatnonzero(ebits == 0)
+        ecol = ef.col.astype(np.int64)
+        for s in range(S):
+            gb0 = 0 if s * csr.m + r0 == 0 else int(far_stop[s * csr.m + r0 - 1]) + 1
+            gb1 = int(far_stop[s * csr.m + r1 - 1]) + 1
+            wb0 = 0 if s * sub.m == 0 else int(estop[s * sub.m - 1]) + 1
+            wb1 = int(estop[s * sub.m + sub.m - 1]) + 1
+            assert gb1 - gb0 == wb1 - wb0
+            k0, k1 = gb0 // TCf, -(-gb1 // TCf)
+            off = gb0 - k0 * TCf
+            fl = np.unpackbits(A.export_range("flags", k0, k1 - k0), bitorder="little")
+            assert np.array_equal(fl[off: off + gb1 - gb0], ebits[wb0:wb1])
+            col = A.export_range("col", k0, k1 - k0).astype(np.int64)
+            assert np.array_equal(col[off: off + gb1 - gb0], ecol[wb0:wb1])
+            v = A.export_range("val0", k0, k1 - k0).view(np.uint32)
+            assert np.array_equal(v[off: off + gb1 - gb0], ef.val[0].view(np.uint32)[wb0:wb1])

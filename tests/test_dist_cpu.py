@@ -202,7 +202,7 @@ class _ShmFusedMatrix:
         return 0
 
 
-def _fused_worker(rank, world, port, root, n, iters):
+def _fused_worker(rank, world, port, root, n, iters, restart_after=0):
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -217,6 +217,10 @@ def _fused_worker(rank, world, port, root, n, iters):
     sub.val = sub.val.astype(np.float64)
     pit = D.FusedPowerIteration(L, _ShmFusedMatrix(sub, L.m_local), torch.float64, "cpu",
                                 comm_factory=_ShmComm)
+    if restart_after:  # a few steps, then restart: the peers' last stores must land first
+        for _ in range(restart_after):
+            pit.step()
+        pit.restart()
     for _ in range(iters):
         pit.step()
     x = pit.current_x()
@@ -225,14 +229,16 @@ def _fused_worker(rank, world, port, root, n, iters):
     dist.destroy_process_group()
 
 
-def test_fused_power_iteration_host_protocol_world2():
+@pytest.mark.parametrize("restart_after", [0, 3])
+def test_fused_power_iteration_host_protocol_world2(restart_after):
     """dist.FusedPowerIteration over gloo world 2: IPC-handle exchange in rank order, x_0
     layout, restart barrier, and the parity/epoch protocol of comm.cu (modelled on shared
-    files) give every rank the single-process power iteration."""
+    files) give every rank the single-process power iteration — also after a restart in the
+    middle (the restart waits for every peer's last step before re-initialising x_0)."""
     import torch.multiprocessing as mp
     n, iters, world = 1 << 12, 4, 2
     with tempfile.TemporaryDirectory() as td:
-        mp.spawn(_fused_worker, args=(world, _free_port(), td, n, iters), nprocs=world, join=True)
+        mp.spawn(_fused_worker, args=(world, _free_port(), td, n, iters, restart_after), nprocs=world, join=True)
         xs = [np.load(os.path.join(td, f"x{r}.npy")) for r in range(world)]
     from synth import matrices as sm
     a = sm.circuit_like_rows(0, n, n=n, n_net=2, net_log2=(8, 10), band=512)
@@ -253,7 +259,16 @@ class _FailingOpenComm(_ShmComm):
         super().open_ipc(handles)
 
 
-def _fused_fail_worker(rank, world, port, root, fail_create):
+class _FailingHandleComm(_ShmComm):
+    """Rank 1 cannot export an IPC handle for its buffer."""
+
+    def ipc_handle(self):
+        if self.rank == 1:
+            raise OSError("cudaIpcGetMemHandle failed")
+        return super().ipc_handle()
+
+
+def _fused_fail_worker(rank, world, port, root, fail_create, fail_handle=False):
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -267,7 +282,7 @@ def _fused_fail_worker(rank, world, port, root, fail_create):
     def factory(*a):
         if fail_create and rank == 0:
             raise MemoryError("no device memory for the exchange buffers")
-        return _FailingOpenComm(*a)
+        return _FailingHandleComm(*a) if fail_handle else _FailingOpenComm(*a)
 
     try:
         D.FusedPowerIteration(L, None, torch.float64, "cpu", comm_factory=factory)
@@ -280,13 +295,16 @@ def _fused_fail_worker(rank, world, port, root, fail_create):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("fail_create", [False, True])
-def test_fused_setup_failure_is_agreed_by_every_rank(fail_create):
-    """If one rank cannot create or map the exchange buffers, every rank raises (so bench.py
-    falls back to the NCCL protocol everywhere) instead of the others blocking in a barrier."""
+@pytest.mark.parametrize("mode", ["create", "open", "handle"])
+def test_fused_setup_failure_is_agreed_by_every_rank(mode):
+    """If one rank cannot create, export or map the exchange buffers, every rank raises (so
+    bench.py falls back to the NCCL protocol everywhere) instead of the others blocking in a
+    collective or a barrier."""
     import torch.multiprocessing as mp
     with tempfile.TemporaryDirectory() as td:
-        mp.spawn(_fused_fail_worker, args=(2, _free_port(), td, fail_create), nprocs=2, join=True)
+        mp.spawn(_fused_fail_worker, args=(2, _free_port(), td, mode == "create", mode == "handle"), nprocs=2,
+                 join=True)
         outs = [open(os.path.join(td, f"r{r}.txt")).read() for r in range(2)]
-    want = "create the exchange buffers on rank(s) [0]" if fail_create else "map the peers' buffers on rank(s) [1]"
+    want = {"create": "create the exchange buffers on rank(s) [0]", "open": "map the peers' buffers on rank(s) [1]",
+            "handle": "export the IPC handles on rank(s) [1]"}[mode]
     assert all(want in o for o in outs), outs

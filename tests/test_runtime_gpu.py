@@ -91,7 +91,9 @@ import synth
 from paper_conf_ppopp_yanlzz14_b200 import Matrix
 csr = synth.webbase_like(m=20000)
 x = torch.from_numpy(synth.make_x(csr.n, np.float32, "unit", 0)).cuda()
-for p in (dict(T=4, C=64), dict(T=16, C=256, S=3, empty_mode=2), dict(T=8, C=128, col_mode=3)):
+PLAIN = (dict(T=4, C=64), dict(T=16, C=256, S=3, empty_mode=2), dict(T=8, C=128, col_mode=3),
+         dict(T=4, C=64, tpc=2), dict(T=16, C=128, rc=2), dict(T=8, C=64, rc=2, tpc=2))
+for p in PLAIN + (() if "--plain-only" in sys.argv else (dict(B=1024, R=4096, W=512), dict(B=1024, R=4096, W=512, S=2))):
     A = Matrix.from_synth(csr, device=0, **p)
     A.spmv(x); torch.cuda.synchronize(); A.free()
 c = synth.fem_like("cantilever")
@@ -101,18 +103,24 @@ print("SANITIZE-DONE")
 """ % ROOT
 
 
-@pytest.mark.parametrize("tool", ["memcheck", "synccheck"])
+@pytest.mark.parametrize("tool", ["memcheck", "synccheck", "initcheck", "racecheck"])
 def test_compute_sanitizer(tool, tmp_path):
+    """memcheck / synccheck / initcheck over the plain kernels (incl. tiles_per_cta = 2 and
+    the strategy-2 result cache) and the panel-sliced band kernel; racecheck over the plain
+    kernels (the band kernel's look-back flags are volatile shared-memory polls, which
+    racecheck cannot order)."""
     exe = "/usr/local/cuda/bin/compute-sanitizer"
     if not os.path.exists(exe):
         pytest.skip("compute-sanitizer not available")
     script = tmp_path / "san.py"
     script.write_text(SANITIZE)
-    r = subprocess.run([exe, "--tool", tool, "--error-exitcode", "9", "--kernel-name", "kns=yaspmv",
-                        sys.executable, str(script)], capture_output=True, text=True, timeout=900)
+    extra = ["--plain-only"] if tool == "racecheck" else []
+    args = [exe, "--tool", tool, "--error-exitcode", "9", "--kernel-name", "kns=yaspmv"]
+    r = subprocess.run(args + [sys.executable, str(script)] + extra, capture_output=True, text=True, timeout=1800)
     assert "SANITIZE-DONE" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
     assert r.returncode == 0, r.stdout[-3000:]
-    assert "ERROR SUMMARY: 0 errors" in r.stdout
+    assert ("RACECHECK SUMMARY: 0 hazards" if tool == "racecheck" else "ERROR SUMMARY: 0 errors") in r.stdout, \
+        r.stdout[-3000:]
 
 
 @pytest.mark.parametrize("S", [1, 3])
@@ -202,3 +210,37 @@ def test_ablation_variants_match():
     torch.cuda.synchronize()
     for o in outs:
         assert np.array_equal(o.astype(np.float64), ye)
+
+
+SPIN = r"""
+import ctypes, numpy as np, torch, sys
+sys.path.insert(0, %r)
+from paper_conf_ppopp_yanlzz14_b200 import Matrix
+from paper_conf_ppopp_yanlzz14_b200._lib import lib
+# row 0 holds 600 blocks (tiles of 4 x 64 = 256 blocks: it ends in tile 2), then short rows
+m, n = 2000, 4096
+lens = np.ones(m, dtype=np.int64); lens[0] = 600
+rp = np.zeros(m + 1, dtype=np.int64); np.cumsum(lens, out=rp[1:])
+col = np.concatenate([np.arange(600), np.arange(1, m) %% n]).astype(np.int32)
+A = Matrix.from_csr(m, n, rp, col, np.ones(rp[-1], np.float32), device=0, T=4, C=64, col_mode=2)
+x = torch.ones(n, device="cuda"); y = torch.empty(m, device="cuda")
+st = lib.yaspmv_ablation_spmv(A._h, 12, x.data_ptr(), y.data_ptr(), torch.cuda.current_stream().cuda_stream)
+try:
+    torch.cuda.synchronize()
+    print("NO-TRAP")
+except Exception as e:
+    print("TRAPPED", type(e).__name__)
+print("SPIN-TILE", int(lib.yaspmv_debug_spin_tile()))
+""" % ROOT
+
+
+def test_debug_spin_bound_traps_with_tile_id(tmp_path):
+    """with YASPMV_SPIN_LIMIT set, a look-back whose predecessor never publishes
+    (ablation variant 12: tile 0 skips its publish) traps instead of hanging the GPU, and the
+    waiting tile's id is readable afterwards (tile 2: the stop of the 600-block row)."""
+    script = tmp_path / "spin.py"
+    script.write_text(SPIN)
+    env = dict(os.environ, YASPMV_SPIN_LIMIT="20000")
+    r = subprocess.run([sys.executable, str(script)], capture_output=True, text=True, timeout=300, env=env)
+    assert "TRAPPED" in r.stdout, r.stdout + r.stderr[-2000:]
+    assert "SPIN-TILE 2" in r.stdout, r.stdout
