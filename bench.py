@@ -102,6 +102,28 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(rows)}
 
 
+def bind_numa_local(gpu: int) -> dict:
+    """Run on the CPUs of the GPU's NUMA node, so that pinned host buffers (first touch)
+    are NUMA-local to the GPU for the e2e copies."""
+    try:
+        import torch
+        p = torch.cuda.get_device_properties(gpu)
+        bus = f"{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+        with open(f"/sys/bus/pci/devices/{bus}/numa_node") as f:
+            node = int(f.read().strip())
+        if node < 0:
+            return {"numa_node": None, "note": "no NUMA affinity reported"}
+        with open(f"/sys/devices/system/node/node{node}/cpulist") as f:
+            cpus = set()
+            for part in f.read().strip().split(","):
+                a, _, b = part.partition("-")
+                cpus.update(range(int(a), int(b or a) + 1))
+        os.sched_setaffinity(0, cpus)
+        return {"numa_node": node, "cpus": len(cpus), "pci": bus}
+    except Exception as e:
+        return {"numa_node": None, "note": f"{type(e).__name__}: {e}"[:120]}
+
+
 def measured_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -435,10 +457,24 @@ def main():
     # ---- e2e through the public API with HOST buffers (pinned) -----------------------
     # every step copies x host->device and y device->host; yaspmv_spmv_host_async overlaps
     # the copies of consecutive steps with the SpMV (three buffer slots, two copy streams)
+    numa = bind_numa_local(local_rank % ngpu)  # pinned buffers on the GPU's NUMA node
     xh = torch.empty(L.n_padded, dtype=tdt).pin_memory()
     x_cur = fpit.current_x(stream) if fpit is not None else pit.current_x()
     xh.copy_(x_cur.cpu())
     yh = torch.empty(L.m_local, dtype=tdt).pin_memory()
+    # the copy engines alone: one H2D of x and one D2H of y, CUDA events
+    xd = torch.empty_like(xh, device=dev)
+    yd = torch.empty_like(yh, device=dev)
+    c0, c1, c2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+    c0.record(stream)
+    xd.copy_(xh, non_blocking=True)
+    c1.record(stream)
+    yh.copy_(yd, non_blocking=True)
+    c2.record(stream)
+    torch.cuda.synchronize()
+    h2d_gbs = xh.numel() * xh.element_size() / (c0.elapsed_time(c1) * 1e-3) / 1e9
+    d2h_gbs = yh.numel() * yh.element_size() / (c1.elapsed_time(c2) * 1e-3) / 1e9
+    del xd, yd
     A.spmv_host_async(xh.numpy(), yh.numpy(), stream=stream.cuda_stream)
     A.host_sync()
     if world > 1:
@@ -455,7 +491,11 @@ def main():
            "h2d_bytes_per_step": int(L.n_padded * np.dtype(dtype_np).itemsize * world),
            "d2h_bytes_per_step": int(int(L.bounds[-1]) * np.dtype(dtype_np).itemsize),
            "api": "yaspmv_spmv_host_async + yaspmv_host_sync (pinned x in, y out every step, per rank)",
-           "steps": args.e2e_steps}
+           "steps": args.e2e_steps, "h2d_gbs": h2d_gbs, "d2h_gbs": d2h_gbs, "pinned_numa": numa,
+           # the pipeline overlaps copy-in, SpMV and copy-out of consecutive steps: a step
+           # costs at least the slowest of the three
+           "h2d_ms": L.n_padded * np.dtype(dtype_np).itemsize / h2d_gbs / 1e6,
+           "d2h_ms": L.m_local * np.dtype(dtype_np).itemsize / d2h_gbs / 1e6}
 
     # ---- N > 1: the fused exchange (peer stores from the SpMV epilogue) as extra keys ---
     fused_info = None

@@ -93,7 +93,8 @@ typedef struct {
      ceil((R + 2*band)/W), go to the band stream, whose every gather is served from a
      W-value window of x in shared memory; the rest is a plain BCCOO/BCCOO+ matrix encoded
      with the fields above.  fp32, 1x1 blocks; not with the fused multi-GPU step. */
-  int32_t band;        /* band half-width B in columns; 0 = off (plain format)           */
+  int32_t band;        /* band half-width B in columns; 0 = off (plain format);
+                          yaspmv_reencode: 0 = keep the handle's band fields, -1 = off      */
   int32_t panel_rows;  /* R: multiple of 256, <= 32768; 0 = 16384                        */
   int32_t slice_width; /* W: multiple of 4, <= 65532, KS <= 64; 0 = 16384                */
   int32_t band_col0;   /* column of row 0 (a row-partitioned rank: its first global row) */

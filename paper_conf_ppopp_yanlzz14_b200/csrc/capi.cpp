@@ -788,11 +788,21 @@ yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
   if (!params || !want.flags) want.flags = cur.flags;
   want.rc = want.rc == 0 ? cur.rc : (want.rc < 0 ? 0 : want.rc);
   if (!want.tpc) want.tpc = cur.tpc;
+  // panel-sliced BCCOO+: 0 = keep the handle's band parameters, band = -1 = plain format
+  if (want.band == 0) {
+    want.band = cur.band;
+    if (!want.pR) want.pR = cur.pR;
+    if (!want.pW) want.pW = cur.pW;
+    if (!want.col0) want.col0 = cur.col0;
+  } else if (want.band < 0) {
+    want.band = want.pR = want.pW = want.col0 = 0;
+  }
   {  // only launch-time parameters change (strategy, tiles per CTA): no re-encode
     Params rp;
     if (A->device >= 0 && resolve_params(want, A->csr.m, A->csr.n, rp) == YASPMV_OK && rp.h == cur.h &&
         rp.w == cur.w && rp.S == cur.S && rp.T == cur.T && rp.C == cur.C && rp.col_mode == cur.col_mode &&
-        (rp.empty_mode == 0 || rp.empty_mode == cur.empty_mode) && rp.flags == cur.flags)
+        (rp.empty_mode == 0 || rp.empty_mode == cur.empty_mode) && rp.flags == cur.flags && rp.band == cur.band &&
+        rp.pR == cur.pR && rp.pW == cur.pW && rp.col0 == cur.col0)
       return set_launch(A, rp.rc, rp.tpc);
   }
   return encode_into(A, want);

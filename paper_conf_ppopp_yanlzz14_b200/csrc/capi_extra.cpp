@@ -265,8 +265,11 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   // (1) footprint of every Table-1 block shape; keep the 4 smallest
   struct Shape { int64_t fp; int h, w; };
   std::vector<Shape> shapes;
-  for (int h = 1; h <= 4; ++h)
+  // a panel-sliced BCCOO+ handle tunes its far part (1x1 blocks, band kept by re-encoding)
+  const bool band = A->band_on;
+  for (int h = 1; h <= (band ? 1 : 4); ++h)
     for (int w : {1, 2, 4, 8}) {
+      if (band && w > 1) continue;
       bool any = false;
       for (int T : {4, 8, 16, 32}) any |= find_kernel(A->dtype, h, w, T, COL_I32) != nullptr;
       if (!any) continue;
@@ -282,7 +285,9 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   // (2) candidates: slices only when x is a large share of L2 (BCCOO+ helps x locality,
   // P:154; its temporary buffer costs traffic)
   std::vector<int> Ss = {1};
+  // Table 1's slice counts up to 32; the larger ones only when x is several times L2
   if ((int64_t)M.n * vs * 2 > (int64_t)l2) Ss = {1, 2, 4, 8};
+  if ((int64_t)M.n * vs > 4 * (int64_t)l2) Ss = {1, 2, 4, 8, 16, 32};
 
   // scratch x / y for timing
   void* x = nullptr;
@@ -309,7 +314,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
       for (int cm : cms) {
         // host: one encode per (h, w, S, col mode) at the largest tile, (T, C) variants
         // derived; GPU translation: a full encode per candidate on the device
-        const bool gpu = (saved.flags & YASPMV_GPU_ENCODE) != 0;
+        const bool gpu = (saved.flags & YASPMV_GPU_ENCODE) != 0 || band;
         Params bp0;
         bp0.h = sh.h; bp0.w = sh.w; bp0.S = S; bp0.T = 32; bp0.C = 512; bp0.col_mode = cm;
         bp0.empty_mode = saved.empty_mode;
@@ -326,7 +331,8 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             const int64_t tiles = (nnzb_est + (int64_t)T * C - 1) / ((int64_t)T * C);
             if (tiles < 2 * sms && (T * C) > 1024) continue;
             if (gpu) {
-              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode, YASPMV_GPU_ENCODE, -1, 1};
+              yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode,
+                               (saved.flags & YASPMV_GPU_ENCODE) ? YASPMV_GPU_ENCODE : keep_flags, -1, 1};
               if (yaspmv_reencode(A, &ap) != YASPMV_OK) continue;
             } else {
               Canonical cand;

@@ -170,3 +170,23 @@ def test_host_buffers():
         _check(csr, A.spmv_host(x), x)
     finally:
         A.free()
+
+
+def test_tune_and_reencode_keep_the_band():
+    """yaspmv_tune on a panel-sliced handle tunes its far part (Table 1 over 1x1 blocks) and
+    keeps the band stream; yaspmv_reencode(band = -1) returns to the plain format."""
+    mk, params = CASES["webbase"]
+    csr = mk()
+    x = synth.make_x(csr.n, np.float32, "uniform", 7)
+    A = _build(csr, **params)
+    try:
+        chosen = A.tune()
+        info = A.info()
+        assert info["band_blocks"] > 0 and chosen["block_h"] == chosen["block_w"] == 1
+        assert info["params"]["band"] == params["B"]
+        _check(csr, _run(A, x), x)
+        A.reencode(B=-1)
+        assert A.info()["band_blocks"] == 0
+        _check(csr, _run(A, x), x)
+    finally:
+        A.free()
