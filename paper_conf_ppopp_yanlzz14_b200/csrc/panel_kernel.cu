@@ -50,6 +50,10 @@ __device__ __forceinline__ uint32_t ld_flags16(const uint8_t* p) {
   return v;
 }
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+// acc slot of panel row r (identity: padded or permuted layouts that spread the warp's
+// stops, ~8 rows apart, over the banks cost more address arithmetic than the conflicts they
+// remove — measured 2.26 / 2.43 ms vs 2.15 ms on C5)
+__device__ __forceinline__ int swz(int r) { return r; }
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, unsigned count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
@@ -192,7 +196,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       }
 #pragma unroll
       for (int j = 0; j < 8; ++j)
-        if (r0 + j * NTH < R) acc[r0 + j * NTH] = (VT)s[j];
+        if (r0 + j * NTH < R) acc[swz(r0 + j * NTH)] = (VT)s[j];
     }
   }
   __syncthreads();
@@ -251,6 +255,20 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     fl = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
     trank = __ldg(a.tile_rank + tile);
   };
+  // this warp's tile after (kk, u): the next one of the slice, else its first tile of the
+  // next non-empty slice that has one (kk = KS: none)
+  auto next_tile = [&](int kk, int u) {
+    u += NCW;
+    while (kk < KS && (sh.sp[kk + 1] - sh.sp[kk]) >> 9 <= u) {
+      kk = next_nonempty(kk + 1);
+      u = wid;
+    }
+    return make_int2(kk, u);
+  };
+  if (wid < NCW) {  // the warp's first tile in flight before the first window wait
+    const int2 f = next_tile(k, wid - NCW);
+    if (f.x < KS) load_tile((sh.sp[f.x] >> 9) + f.y);
+  }
   while (k < KS) {
     const int ltile_k = sh.sp[k] >> 9;                     // panel-local first tile of the slice
     const int ntile_k = (sh.sp[k + 1] - sh.sp[k]) >> 9;    // tiles of the slice
@@ -264,7 +282,6 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     bool pending = o > 0;  // X_o still ahead of this warp
     for (int u = wid; u < ntile_k; u += NCW) {
       const int lt = ltile_k + u;       // panel-local tile index (tag of its carry record)
-      load_tile(lt);
       // flow control (slices of more than LAG tiles only): the record slot of this tile
       // must have been released
       if (ntile_k > LAG && u >= LAG) {
@@ -280,25 +297,31 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
         const int c = (int)((cw[i >> 1] >> (16 * (i & 1))) & 0xFFFFu);
         pr[i] = __uint_as_float(vw[i]) * wk[c];
       }
-      // ---- per-thread segmented sum (P:262): pr[i] := sum of its segment up to block i
       const uint32_t stops = ~fl & 0xFFFFu;
+      const int tr = trank;
+      // ---- per-thread segmented sum (P:262): pr[i] := sum of its segment up to block i
       const int nst = __popc(stops);
 #pragma unroll
       for (int i = 1; i < BT; ++i) pr[i] = ((stops >> (i - 1)) & 1u) ? pr[i] : pr[i - 1] + pr[i];
       const VT tail = ((stops >> (BT - 1)) & 1u) ? VT(0) : pr[BT - 1];
-      // ---- warp segmented scan of (has_stop, last partial sum) ----------------
-      int f = nst > 0, nn = nst;
+      // ---- warp segmented scan of (has_stop, last partial sum); the stop count
+      // rides in the low 16 bits and the has-stop flag above (a sum of flags is non-zero
+      // iff their OR is) -----------------------------------------------------------------
+      int fn_ = nst | ((nst > 0) << 16);
       VT v = tail;
 #pragma unroll
       for (int d = 1; d < 32; d <<= 1) {
-        const int f2 = __shfl_up_sync(0xffffffffu, f, d);
-        const int n2 = __shfl_up_sync(0xffffffffu, nn, d);
+        const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
         const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
         if (lane >= d) {
-          if (!f) v = v2 + v;
-          f |= f2;
-          nn += n2;
+          if (!(fn_ >> 16)) v = v2 + v;
+          fn_ += g2;
         }
+      }
+      const int f = (fn_ >> 16) != 0;
+      {  // the warp's next tile in flight during this tile's updates and look-back
+        const int2 nx2 = next_tile(k, u);
+        if (nx2.x < KS) load_tile((sh.sp[nx2.x] >> 9) + nx2.y);
       }
       // ---- publish the tile's carry record (before anything waits on others) ----------
       if (lane == 31) {
@@ -307,8 +330,9 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
         __threadfence_block();
         sh.rtag[lt % RING] = lt + 1;
       }
-      int fx = __shfl_up_sync(0xffffffffu, f, 1);
-      int nx = __shfl_up_sync(0xffffffffu, nn, 1);
+      const int gx = __shfl_up_sync(0xffffffffu, fn_, 1);
+      int fx = (gx >> 16) != 0;
+      int nx = gx & 0xFFFF;
       VT vx = __shfl_up_sync(0xffffffffu, v, 1);
       if (lane == 0) {
         fx = 0;
@@ -325,7 +349,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       // (vx); when it continues earlier tiles (dep) their carry is added below, after the
       // look-back — a fixed association, so y stays bitwise deterministic
       const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
-      const int row_first = frk + trank + nx;
+      const int row_first = frk + tr + nx;
       {
         VT* ar = acc + row_first;
         VT add = vx;
@@ -351,7 +375,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
           }
         }
         carry = __shfl_sync(0xffffffffu, carry, 0);
-        if (dep) acc[row_first] = acc[row_first] + carry;
+        if (dep) acc[swz(row_first)] = acc[swz(row_first)] + carry;
       }
     }
     if (pending) slice_barrier(o);  // no tile of this slice: still part of X_o
@@ -363,7 +387,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   // ---- epilogue: y := acc (scaled), sum of y^2 ----------------------------------------
   const double inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   for (int r = t; r < rows; r += NTH) {
-    const VT o2 = (a.epi & 1) ? (VT)(acc[r] * inv) : acc[r];
+    const VT o2 = (a.epi & 1) ? (VT)(acc[swz(r)] * inv) : acc[swz(r)];
     y[row0 + r] = o2;
     ssq += (double)o2 * (double)o2;
   }
