@@ -206,20 +206,21 @@ def _free_port():
     return p
 
 
-def _ipc_worker(rank, world, port, path, iters):
+def _ipc_worker(rank, world, port, path, iters, per_rank_device=False):
     import torch.distributed as dist
     from synth import matrices as sm
     from paper_conf_ppopp_yanlzz14_b200 import Matrix, dist as D
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    torch.cuda.set_device(0)
+    dev = rank if per_rank_device else 0
+    torch.cuda.set_device(dev)
     csr = sm.circuit_like_rows(0, KW["n"], **KW)
     L = D.make_layout(csr.row_ptr, rank, world)
     sub = csr.row_slice(L.r0, L.r1)
     A = Matrix.from_csr(sub.m, L.n_padded, sub.row_ptr, D.remap_columns(sub.col, L.bounds, L.m_max), sub.val,
-                        device=0, T=16, C=128)
-    pit = D.FusedPowerIteration(L, A, torch.float32, "cuda:0", timeout_ms=60000)  # IPC handle exchange
+                        device=dev, T=16, C=128)
+    pit = D.FusedPowerIteration(L, A, torch.float32, f"cuda:{dev}", timeout_ms=60000)  # IPC handle exchange
     for _ in range(iters):
         pit.step()
     pit.comm.wait()
@@ -233,16 +234,21 @@ def _ipc_worker(rank, world, port, path, iters):
     dist.destroy_process_group()
 
 
-def test_fused_two_processes_ipc_one_gpu():
-    """Two processes mapping each other's comm through CUDA IPC (the multi-GPU code path;
-    here both map cuda:0); the result equals the single-process unfused protocol bitwise."""
+@pytest.mark.parametrize("two_devices", [False, True])
+def test_fused_two_processes_ipc(two_devices):
+    """Two processes mapping each other's comm through CUDA IPC; the result equals the
+    single-process unfused protocol bitwise.  two_devices = False: both map cuda:0 (always
+    runs); True: rank r on cuda:r, so the peer stores, the system-scope fences and the
+    acquire/release flags cross NVLink (runs only where two GPUs are visible)."""
     _need_gpu()
+    if two_devices and torch.cuda.device_count() < 2:
+        pytest.skip("needs two visible GPUs")
     import torch.multiprocessing as mp
     from synth import matrices as sm
     iters = 3
     with tempfile.TemporaryDirectory() as td:
         path = os.path.join(td, "z")
-        mp.spawn(_ipc_worker, args=(2, _free_port(), path, iters), nprocs=2, join=True)
+        mp.spawn(_ipc_worker, args=(2, _free_port(), path, iters, two_devices), nprocs=2, join=True)
         zs = [np.load(path + f".{r}.npy") for r in range(2)]
         n2 = [np.load(path + f".{r}.n2.npy") for r in range(2)]
     csr = sm.circuit_like_rows(0, KW["n"], **KW)
