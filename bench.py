@@ -540,7 +540,9 @@ def main():
         kern = {}
         if prof and prof["calls"]:
             S = info["params"]["slices"]
-            if band:  # far K1 writes its S slice results, the band kernel K4 reads and combines them
+            if band and info["params"]["band_far"] == 2:  # P7: one kernel, far entries in every panel's slice 0
+                kern["panel_kernel (band + far slices)"] = (prof["band_ms"] / prof["calls"], info["alg_bytes"])
+            elif band:  # far K1 writes its S slice results, the band kernel K4 reads and combines them
                 far_bytes = info["format_bytes"] - info["band_format_bytes"] + info["n"] * sv + S * info["m"] * sv
                 kern["spmv_bccoo_kernel (far part)"] = (prof["plain_ms"] / prof["calls"], far_bytes)
                 kern["panel_kernel (band)"] = (prof["band_ms"] / prof["calls"],

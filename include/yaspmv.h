@@ -98,7 +98,19 @@ typedef struct {
   int32_t panel_rows;  /* R: multiple of 256, <= 32768; 0 = 16384                        */
   int32_t slice_width; /* W: multiple of 4, <= 65532, KS <= 64; 0 = 16384                */
   int32_t band_col0;   /* column of row 0 (a row-partitioned rank: its first global row) */
+  int32_t band_far;    /* where the entries outside the band go (reading P7):
+                          YASPMV_FAR_SEPARATE = a plain BCCOO/BCCOO+ matrix run before the
+                          band kernel (its S slices combined in the band kernel's prologue);
+                          YASPMV_FAR_IN_PANEL = slice 0 of every panel: one BCCOO slice over
+                          all n columns with int32 columns, gathered from global memory by
+                          the band kernel itself (one launch per SpMV, no partial vectors;
+                          on C5 its random gathers over all of x miss L2 far more often
+                          than BCCOO+'s column slices: 10.0 vs 3.3 ms).
+                          0 = YASPMV_FAR_SEPARATE; yaspmv_tune times both;
+                          yaspmv_reencode: 0 = keep                                        */
 } yaspmv_params;
+
+enum { YASPMV_FAR_SEPARATE = 1, YASPMV_FAR_IN_PANEL = 2 };
 
 typedef struct {
   int64_t m, n, nnz;         /* matrix shape and structural non-zeros after normalisation */
@@ -129,6 +141,9 @@ typedef struct {
   int64_t band_stops;        /* row stops of the band stream                              */
   int64_t band_format_bytes; /* device bytes of the band stream + its aux read by one SpMV
                                 (included in format_bytes; the far part is the rest)       */
+  int64_t band_far_blocks_pad; /* YASPMV_FAR_IN_PANEL: blocks of the panels' far slices
+                                (incl. FILLER blocks and padding; part of band_blocks_pad);
+                                its entries are nnz - band_blocks                          */
 } yaspmv_info;
 
 /* ---------------------------------------------------------------- build / free
@@ -239,21 +254,28 @@ enum {
   YASPMV_ARR_FLAGS = 0, YASPMV_ARR_COL = 1, YASPMV_ARR_COL_DELTA = 2,
   YASPMV_ARR_VAL0 = 3, YASPMV_ARR_VAL1 = 4, YASPMV_ARR_VAL2 = 5, YASPMV_ARR_VAL3 = 6,
   YASPMV_ARR_SEG_ROW = 7, YASPMV_ARR_ZERO_ROWS = 8, YASPMV_ARR_CTA_SEG0 = 9, YASPMV_ARR_FRE = 10,
-  /* panel-sliced BCCOO+ band stream (params.band > 0; readings P1-P6 of DESIGN.md §2.1):
+  /* panel-sliced BCCOO+ band stream (params.band > 0; readings P1-P7 of DESIGN.md §2.1).
+   * A panel holds NS = KS slices, or NS = KS + 1 with YASPMV_FAR_IN_PANEL, whose slice 0 is
+   * the far slice (reading P7) and whose band slices are 1..KS; F = band_far_blocks_pad:
    *  BAND_FLAGS      uint8 [band_blocks_pad/8]  0 = last block of its row in its slice
-   *  BAND_COL16      uint16 [band_blocks_pad]   column - (p*R + col0 - B) - k*W; W = FILLER
-   *                  block (value 0) of an empty row inside the slice's row range
+   *  BAND_COL16      uint16 [band_blocks_pad - F] band blocks only: column - (p*R + col0 - B)
+   *                  - k*W; W = FILLER block (value 0) of an empty row inside the slice's rows
    *  BAND_VAL        value [band_blocks_pad]
    *  BAND_PANEL_BLK0 int64 [panels + 1]         first block of each panel
-   *  BAND_SLICE_PTR  int32 [panels * (KS+1)]    block offset of slice k inside its panel (padded)
-   *  BAND_STOP_PTR   int32 [panels * (KS+1)]    row stops before slice k inside its panel
-   *  BAND_FIRST_ROW  int32 [panels * KS]        first non-empty row of each slice (the s-th
+   *  BAND_SLICE_PTR  int32 [panels * (NS+1)]    block offset of slice k inside its panel (padded)
+   *  BAND_STOP_PTR   int32 [panels * (NS+1)]    row stops before slice k inside its panel
+   *  BAND_FIRST_ROW  int32 [panels * NS]        first non-empty row of each slice (the s-th
    *                                              row stop of the slice is row first_row + s)
    *  BAND_TILE_RANK  int32 [band_blocks_pad/512] stops before each 512-block tile in its slice
-   *  (every slice is padded to a multiple of 512 blocks = 16 blocks x 32 threads) */
+   *  BAND_FAR_COL    int32 [F]                  far-slice blocks only: column; n = FILLER
+   *  BAND_FAR_BLK0   int64 [panels + 1]         far-slice blocks before each panel
+   *  (every slice is padded to a multiple of 512 blocks = 16 blocks x 32 threads; block b of
+   *  panel p is the (b - far_blk0[p+1])-th BAND_COL16 entry if it belongs to a band slice, the
+   *  (b - band blocks before p)-th BAND_FAR_COL entry if to the far slice) */
   YASPMV_ARR_BAND_FLAGS = 11, YASPMV_ARR_BAND_COL16 = 12, YASPMV_ARR_BAND_VAL = 13,
   YASPMV_ARR_BAND_PANEL_BLK0 = 14, YASPMV_ARR_BAND_SLICE_PTR = 15, YASPMV_ARR_BAND_STOP_PTR = 16,
-  YASPMV_ARR_BAND_FIRST_ROW = 17, YASPMV_ARR_BAND_TILE_RANK = 18
+  YASPMV_ARR_BAND_FIRST_ROW = 17, YASPMV_ARR_BAND_TILE_RANK = 18, YASPMV_ARR_BAND_FAR_COL = 19,
+  YASPMV_ARR_BAND_FAR_BLK0 = 20
 };
 
 /* yaspmv_export: copy canonical array `which` into host_dst (capacity `bytes`).  Returns
@@ -267,7 +289,8 @@ yaspmv_status yaspmv_export_device(yaspmv_matrix A, int32_t which, void* host_ds
 /* yaspmv_export_device_range: as yaspmv_export_device for the workgroup tiles
  * [first_tile, first_tile + ntiles) only (per-block arrays: the tiles' T*C blocks — 512 for the
  * band stream; CTA_SEG0 / BAND_TILE_RANK: those tiles' entries), for checking windows of
- * matrices whose full arrays are too large to copy. */
+ * matrices whose full arrays are too large to copy.  BAND_COL16 / BAND_FAR_COL count tiles
+ * of their own arrays (band-slice tiles / far-slice tiles). */
 yaspmv_status yaspmv_export_device_range(yaspmv_matrix A, int32_t which, int64_t first_tile, int64_t ntiles,
                                          void* host_dst, int64_t bytes, int64_t* nbytes);
 

@@ -22,7 +22,8 @@ ARR = {"flags": 0, "col": 1, "col_delta": 2, "val0": 3, "val1": 4, "val2": 5, "v
        "seg_row": 7, "zero_rows": 8, "cta_seg0": 9, "fre": 10,
        # panel-sliced BCCOO+ band stream
        "band_flags": 11, "band_col16": 12, "band_val": 13, "band_panel_blk0": 14, "band_slice_ptr": 15,
-       "band_stop_ptr": 16, "band_first_row": 17, "band_tile_rank": 18}
+       "band_stop_ptr": 16, "band_first_row": 17, "band_tile_rank": 18, "band_far_col": 19, "band_far_blk0": 20}
+FAR_SEPARATE, FAR_IN_PANEL = 1, 2  # yaspmv_params.band_far (include/yaspmv.h)
 PANEL_BT, PANEL_BC = 16, 32  # band stream tile: 16 blocks x 32 threads (csrc/panel.hpp PANEL_BT, PANEL_WT)
 
 MAX_RANKS = 8  # YASPMV_MAX_RANKS
@@ -47,7 +48,7 @@ class Params(ctypes.Structure):
                 ("thread_tile", ctypes.c_int32), ("cta_size", ctypes.c_int32), ("col_mode", ctypes.c_int32),
                 ("empty_mode", ctypes.c_int32), ("flags", ctypes.c_int32), ("result_cache", ctypes.c_int32),
                 ("tiles_per_cta", ctypes.c_int32), ("band", ctypes.c_int32), ("panel_rows", ctypes.c_int32),
-                ("slice_width", ctypes.c_int32), ("band_col0", ctypes.c_int32)]
+                ("slice_width", ctypes.c_int32), ("band_col0", ctypes.c_int32), ("band_far", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
@@ -65,7 +66,7 @@ class Info(ctypes.Structure):
                 ("tune_candidates", ctypes.c_int32), ("reserved", ctypes.c_int32),
                 ("band_blocks", ctypes.c_int64), ("band_blocks_pad", ctypes.c_int64), ("band_panels", ctypes.c_int64),
                 ("band_slices", ctypes.c_int64), ("band_stops", ctypes.c_int64),
-                ("band_format_bytes", ctypes.c_int64)]
+                ("band_format_bytes", ctypes.c_int64), ("band_far_blocks_pad", ctypes.c_int64)]
 
     def as_dict(self):
         d = {}

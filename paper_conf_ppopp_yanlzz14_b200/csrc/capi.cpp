@@ -101,6 +101,7 @@ Params from_abi(const yaspmv_params* p) {
     q.pR = p->panel_rows;
     q.pW = p->slice_width;
     q.col0 = p->band_col0;
+    q.bfar = p->band_far;
   }
   return q;
 }
@@ -121,6 +122,7 @@ yaspmv_params to_abi(const Params& q) {
   p.panel_rows = q.pR;
   p.slice_width = q.pW;
   p.band_col0 = q.col0;
+  p.band_far = q.bfar;
   return p;
 }
 
@@ -273,9 +275,11 @@ yaspmv_status install_canonical_impl(yaspmv_matrix A, Canonical&& c, int flags) 
 yaspmv_status resolve_band(yaspmv_matrix A, Params& p) {
   if (p.band < 0) return fail(YASPMV_EINVAL, "band must be >= 0");
   if (p.band == 0) {
-    p.pR = p.pW = p.col0 = 0;
+    p.pR = p.pW = p.col0 = p.bfar = 0;
     return YASPMV_OK;
   }
+  if (p.bfar == 0) p.bfar = YASPMV_FAR_SEPARATE;
+  if (p.bfar != YASPMV_FAR_SEPARATE && p.bfar != YASPMV_FAR_IN_PANEL) return fail(YASPMV_EINVAL, "bad band_far");
   if (A->dtype != YASPMV_F32) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ is compiled for fp32");
   if (p.h != 1 || p.w != 1) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ needs 1x1 blocks");
   if (p.pR == 0) p.pR = 16384;  // defaults: one 1024-thread CTA per SM, 205 KB of shared memory
@@ -305,7 +309,8 @@ yaspmv_status panel_to_device(yaspmv_matrix A, const PanelCanonical& pc, PanelDe
   };
   const int64_t ntl = pc.nband_pad / PANEL_TC;
   yaspmv_status st;
-  if ((st = upload_permuted(reinterpret_cast<const uint8_t*>(pc.col16.data()), ntl, PANEL_WT, 2 * PANEL_BT,
+  if ((st = upload_permuted(reinterpret_cast<const uint8_t*>(pc.col16.data()), (pc.nband_pad - pc.nfar_pad) / PANEL_TC,
+                            PANEL_WT, 2 * PANEL_BT,
                             &nd.col16)) != YASPMV_OK ||
       (st = upload_permuted(pc.val.data(), ntl, PANEL_WT, PANEL_BT * A->vsize, &nd.val)) != YASPMV_OK ||
       (st = up(pc.tile_rank.data(), pc.tile_rank.size() * 4, (void**)&nd.tile_rank)) != YASPMV_OK ||
@@ -313,7 +318,10 @@ yaspmv_status panel_to_device(yaspmv_matrix A, const PanelCanonical& pc, PanelDe
       (st = up(pc.panel_blk0.data(), pc.panel_blk0.size() * 8, (void**)&nd.panel_blk0)) != YASPMV_OK ||
       (st = up(pc.slice_ptr.data(), pc.slice_ptr.size() * 4, (void**)&nd.slice_ptr)) != YASPMV_OK ||
       (st = up(pc.stop_ptr.data(), pc.stop_ptr.size() * 4, (void**)&nd.stop_ptr)) != YASPMV_OK ||
-      (st = up(pc.first_row.data(), pc.first_row.size() * 4, (void**)&nd.first_row)) != YASPMV_OK) {
+      (st = up(pc.first_row.data(), pc.first_row.size() * 4, (void**)&nd.first_row)) != YASPMV_OK ||
+      (st = upload_permuted(reinterpret_cast<const uint8_t*>(pc.far_col.data()), pc.nfar_pad / PANEL_TC, PANEL_WT,
+                            4 * PANEL_BT, &nd.far_col)) != YASPMV_OK ||
+      (st = up(pc.far_blk0.data(), pc.far_blk0.size() * 8, (void**)&nd.far_blk0)) != YASPMV_OK) {
     nd.free_all();
     return st;
   }
@@ -333,6 +341,21 @@ yaspmv_status panel_to_device(yaspmv_matrix A, const PanelCanonical& pc, PanelDe
 }
 
 yaspmv_status encode_plain_into(yaspmv_matrix A, const CSR& src, const Params& p, double t0);
+
+// the plain part of a YASPMV_FAR_IN_PANEL handle: shape only (no blocks, tiles or arrays)
+yaspmv_status install_empty_plain(yaspmv_matrix A, const CSR& src, const Params& p) {
+  Canonical c;
+  c.m = src.m;
+  c.n = src.n;
+  c.MB = src.m;
+  c.NB = src.n;
+  c.SW = std::max<int64_t>(src.n, 1);
+  c.p = p;
+  c.p.h = c.p.w = c.p.S = 1;
+  c.p.empty_mode = EMPTY_FILLER;
+  c.vsize = A->vsize;
+  return install_canonical_impl(A, std::move(c), p.flags);
+}
 
 // (re-)encode A->csr with params and upload; on failure A is left unchanged
 yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
@@ -356,6 +379,7 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
   g.W = p.pW;
   g.B = p.band;
   g.col0 = p.col0;
+  g.fip = p.bfar == YASPMV_FAR_IN_PANEL ? 1 : 0;
   CSR far;
   PanelCanonical pc;
   if ((st = encode_panel(A->csr, g, far, pc)) != YASPMV_OK) return st;
@@ -364,7 +388,8 @@ yaspmv_status encode_into(yaspmv_matrix A, const Params& want) {
     CUDA_TRY(cudaSetDevice(A->device));
     if ((st = panel_to_device(A, pc, nd)) != YASPMV_OK) return st;
   }
-  if ((st = encode_plain_into(A, far, p, t0)) != YASPMV_OK) {
+  // P7: no far part — the plain encoding is an empty m x n matrix (no tiles, no launch)
+  if ((st = g.fip ? install_empty_plain(A, far, p) : encode_plain_into(A, far, p, t0)) != YASPMV_OK) {
     nd.free_all();
     return st;
   }
@@ -456,9 +481,12 @@ yaspmv_status check_device(int32_t device) {
 int64_t band_format_bytes(const yaspmv_matrix A) {
   if (!A->band_on) return 0;
   const PanelCanonical& q = A->pan;
-  int64_t b = q.nband_pad * (int64_t)(A->vsize + 2) + q.nband_pad / 8;
-  b += (q.g.npanels + 1) * 8 + q.g.npanels * (q.g.KS + 1) * 4 + q.g.npanels * q.g.KS * 4;  // panel/slice ptr, first_row
-  b += q.nband_pad / PANEL_TC * 4;  // tile_rank
+  const int64_t NS = q.g.NS();
+  int64_t b = q.nband_pad * (int64_t)A->vsize + q.nband_pad / 8;           // values, flags
+  b += (q.nband_pad - q.nfar_pad) * 2 + q.nfar_pad * 4;                     // col16, far columns (P7)
+  b += (q.g.npanels + 1) * 8 * (q.g.fip ? 2 : 1);                           // panel_blk0 (+ far_blk0)
+  b += q.g.npanels * (NS + 1) * 4 + q.g.npanels * NS * 4;                   // slice_ptr, first_row
+  b += q.nband_pad / PANEL_TC * 4;                                          // tile_rank
   return b;
 }
 
@@ -480,6 +508,7 @@ int64_t alg_bytes(const yaspmv_matrix A) {
   const Params& p = c.p;
   int64_t b = format_bytes(A) + c.n * A->vsize;  // + x
   const int64_t part = (int64_t)p.S * c.MB * p.h * A->vsize;  // far part's output: y or the S slices
+  if (A->band_on && A->pan.g.fip) return b + c.m * A->vsize;  // + y (one kernel, no partials)
   if (A->band_on) return b + part + part + c.m * A->vsize;   // written, re-read by the band kernel, + y
   if (p.S == 1) b += c.m * A->vsize;             // + y
   else b += part + (int64_t)p.S * c.m * A->vsize + c.m * A->vsize;
@@ -621,10 +650,14 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   }
   DeviceGuard dg(A->device);
   if (ev) cudaEventRecord(ev[0], cs);
-  // far part: BCCOO+ slices stay in tmp, the band kernel combines them (no combine kernel)
-  const bool fold = A->can.p.S > 1 && A->can.ntiles > 0;
-  yaspmv_status st = run_spmv_plain(A, x, y, stream, nullptr, nullptr, 0, nullptr, fold);
-  if (st != YASPMV_OK) return st;
+  // far part: BCCOO+ slices stay in tmp, the band kernel combines them (no combine kernel);
+  // P7: the far entries are the panels' slice 0 — no far launch, acc starts at 0
+  const bool fip = A->pan.g.fip != 0;
+  const bool fold = !fip && A->can.p.S > 1 && A->can.ntiles > 0;
+  if (!fip) {
+    yaspmv_status st = run_spmv_plain(A, x, y, stream, nullptr, nullptr, 0, nullptr, fold);
+    if (st != YASPMV_OK) return st;
+  }
   if (ev) cudaEventRecord(ev[1], cs);
   const PanelGeom& g = A->pan.g;
   PanelArgs pa;
@@ -638,8 +671,11 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   pa.tile_rank = A->pd.tile_rank;
   pa.x = x;
   pa.y = y;
+  pa.far_col = A->pd.far_col;
+  pa.far_blk0 = A->pd.far_blk0;
+  pa.fip = fip ? 1 : 0;
   pa.init = fold ? A->d.tmp : y;
-  pa.ninit = fold ? A->can.p.S : 1;
+  pa.ninit = fip ? 0 : fold ? A->can.p.S : 1;
   pa.init_stride = A->can.MB * A->can.p.h;
   pa.m = A->can.m;
   pa.n = A->can.n;
@@ -647,7 +683,7 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   pa.W = g.W;
   pa.B = g.B;
   pa.col0 = g.col0;
-  pa.KS = g.KS;
+  pa.KS = g.NS();
   pa.npanels = g.npanels;
   pa.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
   pa.in_norm2 = in_norm2;
@@ -794,15 +830,17 @@ yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
     if (!want.pR) want.pR = cur.pR;
     if (!want.pW) want.pW = cur.pW;
     if (!want.col0) want.col0 = cur.col0;
+    if (!want.bfar) want.bfar = cur.bfar;
   } else if (want.band < 0) {
-    want.band = want.pR = want.pW = want.col0 = 0;
+    want.band = want.pR = want.pW = want.col0 = want.bfar = 0;
   }
   {  // only launch-time parameters change (strategy, tiles per CTA): no re-encode
     Params rp;
     if (A->device >= 0 && resolve_params(want, A->csr.m, A->csr.n, rp) == YASPMV_OK && rp.h == cur.h &&
         rp.w == cur.w && rp.S == cur.S && rp.T == cur.T && rp.C == cur.C && rp.col_mode == cur.col_mode &&
         (rp.empty_mode == 0 || rp.empty_mode == cur.empty_mode) && rp.flags == cur.flags && rp.band == cur.band &&
-        rp.pR == cur.pR && rp.pW == cur.pW && rp.col0 == cur.col0)
+        rp.pR == cur.pR && rp.pW == cur.pW && rp.col0 == cur.col0 &&
+        (rp.band == 0 || (rp.bfar ? rp.bfar : (int)YASPMV_FAR_SEPARATE) == cur.bfar))
       return set_launch(A, rp.rc, rp.tpc);
   }
   return encode_into(A, want);
@@ -898,6 +936,7 @@ yaspmv_status yaspmv_host_sync(yaspmv_matrix A) {
 int32_t yaspmv_launches_per_spmv(yaspmv_matrix A) {
   if (!A || A->can.m == 0) return 0;
   const int band = A->band_on && A->pan.g.npanels > 0 ? 1 : 0;
+  if (A->band_on && A->pan.g.fip) return band;  // the band kernel alone (P7)
   if (A->can.ntiles == 0) return band;  // memset (+ the band kernel)
   if (band) return 2;                   // far part (its slices combined by the band kernel) + band
   return A->can.p.S > 1 ? 2 : 1;
@@ -983,6 +1022,7 @@ yaspmv_status yaspmv_get_info(yaspmv_matrix A, yaspmv_info* o) {
     o->band_blocks_pad = A->pan.nband_pad;
     o->band_panels = A->pan.g.npanels;
     o->band_slices = A->pan.g.KS;
+    o->band_far_blocks_pad = A->pan.nfar_pad;
     o->band_stops = A->pan.n_stops;
     o->band_format_bytes = band_format_bytes(A);
   }

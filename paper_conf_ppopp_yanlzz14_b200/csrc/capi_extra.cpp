@@ -108,10 +108,13 @@ yaspmv_status describe(yaspmv_matrix A, int which, ArrDesc& d) {
       d.bytes = c.ntiles * p.C * 4;
       break;
     default: {
-      if (which < YASPMV_ARR_BAND_FLAGS || which > YASPMV_ARR_BAND_TILE_RANK) return fail(YASPMV_EINVAL, "unknown array id");
+      if (which < YASPMV_ARR_BAND_FLAGS || which > YASPMV_ARR_BAND_FAR_BLK0) return fail(YASPMV_EINVAL, "unknown array id");
       if (!A->band_on) return fail(YASPMV_EINVAL, "no band stream: the handle is not panel-sliced (band = 0)");
       const PanelCanonical& q = A->pan;
       const PanelGeom& g = q.g;
+      const int64_t NS = g.NS();
+      if ((which == YASPMV_ARR_BAND_FAR_COL || which == YASPMV_ARR_BAND_FAR_BLK0) && !g.fip)
+        return fail(YASPMV_EINVAL, "no far slices: the handle's band_far is YASPMV_FAR_SEPARATE");
       d.band = true;
       d.ntiles = q.nband_pad / PANEL_TC;
       d.C = PANEL_WT;
@@ -119,18 +122,26 @@ yaspmv_status describe(yaspmv_matrix A, int which, ArrDesc& d) {
         case YASPMV_ARR_BAND_FLAGS:
           d.bytes = q.nband_pad / 8; d.host = q.flags.data(); d.dev = A->pd.flags; break;
         case YASPMV_ARR_BAND_COL16:
-          d.bytes = q.nband_pad * 2; d.host = q.col16.data(); d.dev = A->pd.col16; d.ptb = 2 * PANEL_BT; break;
+          d.bytes = (q.nband_pad - q.nfar_pad) * 2; d.host = q.col16.data(); d.dev = A->pd.col16; d.ptb = 2 * PANEL_BT;
+          d.ntiles = (q.nband_pad - q.nfar_pad) / PANEL_TC;
+          break;
+        case YASPMV_ARR_BAND_FAR_COL:
+          d.bytes = q.nfar_pad * 4; d.host = q.far_col.data(); d.dev = A->pd.far_col; d.ptb = 4 * PANEL_BT;
+          d.ntiles = q.nfar_pad / PANEL_TC;
+          break;
+        case YASPMV_ARR_BAND_FAR_BLK0:
+          d.bytes = (g.npanels + 1) * 8; d.host = q.far_blk0.data(); d.dev = A->pd.far_blk0; break;
         case YASPMV_ARR_BAND_VAL:
           d.bytes = q.nband_pad * A->vsize; d.host = q.val.data(); d.dev = A->pd.val; d.ptb = PANEL_BT * A->vsize;
           break;
         case YASPMV_ARR_BAND_PANEL_BLK0:
           d.bytes = (g.npanels + 1) * 8; d.host = q.panel_blk0.data(); d.dev = A->pd.panel_blk0; break;
         case YASPMV_ARR_BAND_SLICE_PTR:
-          d.bytes = g.npanels * (g.KS + 1) * 4; d.host = q.slice_ptr.data(); d.dev = A->pd.slice_ptr; break;
+          d.bytes = g.npanels * (NS + 1) * 4; d.host = q.slice_ptr.data(); d.dev = A->pd.slice_ptr; break;
         case YASPMV_ARR_BAND_STOP_PTR:
-          d.bytes = g.npanels * (g.KS + 1) * 4; d.host = q.stop_ptr.data(); d.dev = A->pd.stop_ptr; break;
+          d.bytes = g.npanels * (NS + 1) * 4; d.host = q.stop_ptr.data(); d.dev = A->pd.stop_ptr; break;
         case YASPMV_ARR_BAND_FIRST_ROW:
-          d.bytes = g.npanels * g.KS * 4; d.host = q.first_row.data(); d.dev = A->pd.first_row; break;
+          d.bytes = g.npanels * NS * 4; d.host = q.first_row.data(); d.dev = A->pd.first_row; break;
         default:
           d.bytes = q.nband_pad / PANEL_TC * 4; d.host = q.tile_rank.data(); d.dev = A->pd.tile_rank; break;
       }
@@ -214,7 +225,7 @@ yaspmv_status yaspmv_export_device_range(yaspmv_matrix A, int32_t which, int64_t
   int64_t tb = 0, total_tiles = 0;
   const bool band = which >= YASPMV_ARR_BAND_FLAGS;
   const int64_t TC = band ? PANEL_TC : (int64_t)c.p.T * c.p.C;
-  const int64_t ntl = band ? A->pan.nband_pad / PANEL_TC : c.ntiles;
+  const int64_t ntl = band ? (d.ntiles >= 0 ? d.ntiles : A->pan.nband_pad / PANEL_TC) : c.ntiles;
   switch (which) {
     case YASPMV_ARR_FLAGS:
     case YASPMV_ARR_BAND_FLAGS: tb = TC / 8; break;
@@ -227,6 +238,7 @@ yaspmv_status yaspmv_export_device_range(yaspmv_matrix A, int32_t which, int64_t
     case YASPMV_ARR_VAL2:
     case YASPMV_ARR_VAL3:
     case YASPMV_ARR_BAND_COL16:
+    case YASPMV_ARR_BAND_FAR_COL:
     case YASPMV_ARR_BAND_VAL: tb = ntl > 0 ? d.bytes / ntl : 0; break;
     default: return fail(YASPMV_EINVAL, "range export: per-block or per-tile arrays only");
   }
@@ -300,11 +312,40 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   cudaEventCreate(&e1);
   cudaStream_t st = (cudaStream_t)stream;
 
-  struct Cand { float ms; int64_t bytes; Params p; };
+  struct Cand { float ms; int64_t bytes; Params p; int bfar; };
   std::vector<Cand> results;
   int results_extra = 0;
   const Params saved = A->can.p;
   const int keep_flags = saved.flags & ~YASPMV_DROP_CSR;
+  auto time_spmv = [&]() {  // median of 7 after 3 warm-up calls (< 0: a call failed)
+    for (int it = 0; it < 3; ++it)
+      if (yaspmv_spmv(A, x, y, stream) != YASPMV_OK) return -1.0f;
+    std::vector<float> ts;
+    for (int it = 0; it < 7; ++it) {
+      cudaEventRecord(e0, st);
+      yaspmv_spmv(A, x, y, stream);
+      cudaEventRecord(e1, st);
+      cudaEventSynchronize(e1);
+      float ms = 0;
+      cudaEventElapsedTime(&ms, e0, e1);
+      ts.push_back(ms);
+    }
+    std::sort(ts.begin(), ts.end());
+    return ts[ts.size() / 2];
+  };
+  // a band handle also times its far entries inside the panels (reading P7) against every
+  // separate far-part candidate below
+  if (band) {
+    yaspmv_params ap{saved.h, saved.w, saved.S, saved.T, saved.C, saved.col_mode, saved.empty_mode, keep_flags,
+                     -1, 1};
+    ap.band_far = YASPMV_FAR_IN_PANEL;
+    if (yaspmv_reencode(A, &ap) == YASPMV_OK) {
+      const float ms = time_spmv();
+      yaspmv_info info;
+      yaspmv_get_info(A, &info);
+      if (ms >= 0) results.push_back({ms, info.format_bytes, A->can.p, YASPMV_FAR_IN_PANEL});
+    }
+  }
   for (const Shape& sh : shapes) {
     const int64_t NB = (M.n + sh.w - 1) / sh.w;
     std::vector<int> cms = {NB < 65535 ? (int)COL_U16 : (int)COL_I32};
@@ -333,6 +374,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             if (gpu) {
               yaspmv_params ap{sh.h, sh.w, S, T, C, cm, saved.empty_mode,
                                (saved.flags & YASPMV_GPU_ENCODE) ? YASPMV_GPU_ENCODE : keep_flags, -1, 1};
+              if (band) ap.band_far = YASPMV_FAR_SEPARATE;
               if (yaspmv_reencode(A, &ap) != YASPMV_OK) continue;
             } else {
               Canonical cand;
@@ -355,7 +397,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
             std::sort(ts.begin(), ts.end());
             yaspmv_info info;
             yaspmv_get_info(A, &info);
-            results.push_back({ts[ts.size() / 2], info.format_bytes, A->can.p});
+            results.push_back({ts[ts.size() / 2], info.format_bytes, A->can.p, A->can.p.bfar});
             // strategy 2 with the paper's pinned result cache sizes 1 and 2: a
             // launch-time switch on the same encoding
             for (int rc : {1, 2}) {
@@ -374,7 +416,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
                   t2.push_back(ms);
                 }
                 std::sort(t2.begin(), t2.end());
-                results.push_back({t2[t2.size() / 2], info.format_bytes, A->can.p});
+                results.push_back({t2[t2.size() / 2], info.format_bytes, A->can.p, A->can.p.bfar});
               }
               set_launch(A, 0, 1);
             }
@@ -393,6 +435,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
     release();
     yaspmv_params back{saved.h, saved.w, saved.S, saved.T, saved.C, saved.col_mode, saved.empty_mode, keep_flags,
                        saved.rc > 0 ? saved.rc : -1, saved.tpc};
+    back.band_far = saved.bfar;
     yaspmv_reencode(A, &back);
     return fail(YASPMV_EUNSUPPORTED, "no tunable candidate could be launched");
   }
@@ -408,6 +451,7 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   }
   yaspmv_params bp{best->p.h, best->p.w, best->p.S, best->p.T, best->p.C, best->p.col_mode, best->p.empty_mode,
                    keep_flags, best->p.rc > 0 ? best->p.rc : -1, 1};
+  bp.band_far = best->bfar;
   yaspmv_status rs = yaspmv_reencode(A, &bp);
   if (rs != YASPMV_OK) {
     release();
@@ -447,6 +491,11 @@ yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chose
   if (chosen) {
     const Params& q = A->can.p;
     *chosen = yaspmv_params{q.h, q.w, q.S, q.T, q.C, q.col_mode, q.empty_mode, q.flags, q.rc, A->tpc};
+    chosen->band = q.band;
+    chosen->panel_rows = q.pR;
+    chosen->slice_width = q.pW;
+    chosen->band_col0 = q.col0;
+    chosen->band_far = q.bfar;
   }
   return YASPMV_OK;
 }

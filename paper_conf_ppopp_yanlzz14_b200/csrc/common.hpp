@@ -41,6 +41,7 @@ struct Params {
   // panel-sliced BCCOO+ (panel.hpp): band half-width (0 = plain format), panel rows,
   // slice width, column of row 0
   int band = 0, pR = 0, pW = 0, col0 = 0;
+  int bfar = 0;  // YASPMV_FAR_SEPARATE / YASPMV_FAR_IN_PANEL (0: resolved by resolve_band)
 };
 
 inline int col_bytes(int mode) { return mode == COL_I32 ? 4 : 2; }

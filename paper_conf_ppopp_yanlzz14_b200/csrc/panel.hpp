@@ -32,25 +32,32 @@ constexpr int PANEL_NBUF = 2;         // x windows resident per CTA (current + n
 
 struct PanelGeom {
   int64_t R = 0, W = 0, B = 0, col0 = 0;  // panel rows, slice width, band half-width, column of row 0
-  int64_t KS = 0;                         // slices per panel = ceil((R + 2B) / W)
+  int64_t KS = 0;                         // band slices per panel = ceil((R + 2B) / W)
   int64_t npanels = 0;
+  int fip = 0;                            // 1: far entries as slice 0 of every panel (reading P7)
+  int64_t NS() const { return KS + fip; } // slices per panel
 };
 
 // host arrays (canonical layout, like Canonical for the plain format)
 struct PanelCanonical {
   PanelGeom g;
   int64_t nband = 0, nfill = 0, nband_pad = 0, n_stops = 0;
+  int64_t nfar_pad = 0;             // P7: blocks of the far slices (incl. fillers and padding)
   std::vector<uint8_t> flags;       // nband_pad / 8, LSB-first, 0 = last entry of its row in its slice
-  std::vector<uint16_t> col16;      // nband_pad: column - cb(p) - k*W (W: FILLER block)
+  std::vector<uint16_t> col16;      // nband_pad - nfar_pad band blocks: column - cb(p) - k*W (W: FILLER)
+  std::vector<int32_t> far_col;     // P7: nfar_pad far-slice blocks: column (n: FILLER block)
+  std::vector<int64_t> far_blk0;    // P7: npanels + 1, far-slice blocks before each panel
   std::vector<uint8_t> val;         // nband_pad values (raw bytes)
   std::vector<int64_t> panel_blk0;  // npanels + 1
-  std::vector<int32_t> slice_ptr;   // npanels * (KS + 1)
-  std::vector<int32_t> stop_ptr;    // npanels * (KS + 1)
-  std::vector<int32_t> first_row;   // npanels * KS: first non-empty row of each slice (panel-relative)
+  std::vector<int32_t> slice_ptr;   // npanels * (NS + 1)
+  std::vector<int32_t> stop_ptr;    // npanels * (NS + 1)
+  std::vector<int32_t> first_row;   // npanels * NS: first non-empty row of each slice (panel-relative)
   std::vector<int32_t> tile_rank;   // nband_pad / TC: stops before each tile inside its slice
   void release_arrays() {
     std::vector<uint8_t>().swap(flags);
     std::vector<uint16_t>().swap(col16);
+    std::vector<int32_t>().swap(far_col);
+    std::vector<int64_t>().swap(far_blk0);
     std::vector<uint8_t>().swap(val);
     std::vector<int64_t>().swap(panel_blk0);
     std::vector<int32_t>().swap(slice_ptr);
@@ -69,6 +76,8 @@ struct PanelDev {
   int32_t* stop_ptr = nullptr;
   int32_t* first_row = nullptr;
   int32_t* tile_rank = nullptr;
+  void* far_col = nullptr;      // P7: device layout (tile transpose), int32
+  int64_t* far_blk0 = nullptr;  // P7
   double* part = nullptr;       // per panel: sum of y^2 (power-iteration epilogue)
   double* scratch = nullptr;
   void free_all();
@@ -88,6 +97,9 @@ struct PanelArgs {
   const int32_t* stop_ptr;
   const int32_t* first_row;
   const int32_t* tile_rank;
+  const void* far_col;       // P7 (fip): int32 columns of the far-slice blocks, device layout
+  const int64_t* far_blk0;   // P7 (fip): far-slice blocks before each panel
+  int fip;                   // 1: slice 0 of every panel is its far slice (KS counts it)
   const void* x;
   void* y;            // out: y = A x (scaled by the epilogue)
   // the far part's result: ninit partial vectors init + s * init_stride (s < ninit), summed in

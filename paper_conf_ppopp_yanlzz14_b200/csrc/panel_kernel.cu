@@ -2,12 +2,14 @@
 // §6.6).  One CTA per row panel of R rows (PAPER.md's workgroup, walking the
 // panel's band stream in workgroup-level tiles of BT*BC blocks):
 //
-//   prologue  acc[0..R) := y[panel rows] (the far part's result, already in y); the
-//             panel's slice offsets to shared memory; the x window of the first slice
-//             (W values, plus the slice's row-occupancy bitmap) requested with
-//             cp.async.bulk on an mbarrier — the part of x one BCCOO+ slice uses,
-//             staged in shared memory so that every gather of the slice is an LDS instead
-//             of a 32-byte L2 request;
+//   prologue  acc[0..R) := the far part's result (its S slice vectors summed in fp64), or
+//             0 when the far entries are the panel's slice 0 (reading P7); the panel's
+//             slice offsets to shared memory; the x windows of the first two band slices
+//             (W values each) requested with cp.async.bulk on an mbarrier — the part of x
+//             one BCCOO+ slice uses, staged in shared memory so that every gather
+//             of the slice is an LDS instead of a 32-byte L2 request;
+//   P7        the far slice first: the same tiles with int32 columns, x gathered from
+//             global memory (its latency overlaps the window loads and the other warps);
 //   per slice the next slice's window is requested into the other buffer; the slice's
 //             workgroup-level tiles (16 blocks x 32 threads = one warp; every slice is
 //             padded to whole tiles, reading P4) go round-robin to the warps, which run
@@ -17,9 +19,9 @@
 //             segmented scan of (has_stop, last partial sum), and the carry into
 //             the tile's first segment by adjacent synchronization with the slice's
 //             earlier tiles — a decoupled look-back over per-tile records in shared
-//             memory; every segment sum is added to acc[row], the row found
-//             through the slice's occupancy bitmap from the tile's first-result entry
-//             (reading P6).  Inside a slice every row has one segment, so no
+//             memory that stops at the nearest final carry-out; every segment
+//             sum is added to acc[row], row = the slice's first row + the stop's rank
+//             from the tile's first-result entry (reading P6).  Inside a slice every row has one segment, so no
 //             two warps touch one row; a barrier between slices keeps each row's slice
 //             sums in ascending order (the BCCOO+ combine order) — deterministic;
 //   epilogue  y[panel rows] := acc (optionally scaled; per-panel sum of y^2).
@@ -95,35 +97,38 @@ struct Layout {
 
 constexpr int NTH = PANEL_CTA, NWARP = NTH / 32, RING = 512, LAG = 128;
 static_assert(PANEL_TC == 512, "tile index = block offset >> 9");
+static_assert(RING > 2 * LAG + NWARP, "a look-back never reads a record slot that was reused");
 
 struct PanelShared {
-  int sp[PANEL_MAX_KS + 1];        // slice_ptr of the panel
-  int fr[PANEL_MAX_KS];            // first_row of every slice
+  int sp[PANEL_MAX_KS + 2];        // slice_ptr of the panel (NS + 1 entries)
+  int fr[PANEL_MAX_KS + 1];        // first_row of every slice
   uint64_t bar[PANEL_NBUF];
-  volatile int armed[PANEL_NBUF];  // window (non-empty slice ordinal) armed on each buffer
-  // carry records of the panel's tiles (decoupled look-back): the tile's last
-  // partial sum and whether it holds a row stop, published before the tag (tile + 1)
+  volatile int armed[PANEL_NBUF];  // window (non-empty band slice ordinal) armed on each buffer
+  // carry records of the panel's tiles (decoupled look-back): rT = the tile's
+  // aggregate (the tail after its last row stop, or its whole sum when it has none), rI =
+  // its carry-out (= rT for a tile holding a stop or starting its slice, carry-in + rT
+  // otherwise); tag 2(t+1): rT published, 2(t+1)+1: rI final as well
   float rT[RING];
-  int rH[RING];
+  float rI[RING];
   volatile int rtag[RING];
   double ss[NWARP];
 };
 
-// Thread 0 requests the x window of the o-th non-empty slice of the panel (its slice id
-// found from the slice offsets) into buffer o % NBUF: W values of x from column cb + k*W
-// with cp.async.bulk on the buffer's mbarrier, the unaligned ends by plain loads, and the
-// zero slot behind the window (the column of a FILLER block, reading P6).
+// Thread 0 requests the x window of the o-th non-empty band slice of the panel (slices
+// kb0..KS-1; its slice id found from the slice offsets) into buffer o % NBUF: W values of x
+// from column cb + (k - kb0)*W with cp.async.bulk on the buffer's mbarrier, the unaligned
+// ends by plain loads, and the zero slot behind the window (a FILLER block's column, P6).
 template <typename VT>
 __device__ __forceinline__ void issue_window(PanelShared& sh, unsigned char* bufs, int64_t bufbytes, const VT* x,
-                                          int64_t n, int64_t xe, int64_t cb, int W, int KS, int o) {
-  int k = 0, oo = -1;
+                                          int64_t n, int64_t xe, int64_t cb, int W, int KS, int kb0, int o) {
+  int k = kb0, oo = -1;
   for (; k < KS; ++k)
     if (sh.sp[k] != sh.sp[k + 1] && ++oo == o) break;
   if (k >= KS) return;
   uint64_t* bar = &sh.bar[o % PANEL_NBUF];
   if (o >= PANEL_NBUF) mbar_wait(bar, (unsigned)((o / PANEL_NBUF - 1) & 1));  // previous use landed
   VT* w = reinterpret_cast<VT*>(bufs + (o % PANEL_NBUF) * bufbytes);
-  const int64_t base = cb + (int64_t)k * W;
+  const int64_t base = cb + (int64_t)(k - kb0) * W;
   const int sh_k = (int)(((xe + base) % 4 + 4) % 4);
   const int64_t lo = max((int64_t)0, base), hi = min(n, base + W);
   unsigned tx = 0;
@@ -149,7 +154,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   __shared__ PanelShared sh;
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
   const int64_t p = blockIdx.x;
-  const int R = (int)a.R, W = (int)a.W, KS = (int)a.KS;
+  const int R = (int)a.R, W = (int)a.W, KS = (int)a.KS, fip = a.fip;
   const Layout L(a.R, a.W);
   VT* acc = reinterpret_cast<VT*>(dsm);
   unsigned char* bufs = dsm + (int64_t)R * sizeof(VT);
@@ -159,9 +164,10 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   const VT* x = static_cast<const VT*>(a.x);
   VT* y = static_cast<VT*>(a.y);
   const int64_t xe = (int64_t)(reinterpret_cast<uintptr_t>(x) / sizeof(VT));
-  // window of slice k: columns [cb + k*W, cb + (k+1)*W); element j of the window sits at
-  // win[shift(k) + j], shift chosen so that shared and global addresses agree mod 16 B
-  auto shift_of = [&](int k) { return (int)(((xe + cb + (int64_t)k * W) % 4 + 4) % 4); };
+  // window of band slice k (slice k - fip of the band): columns [cb + (k-fip)*W, + W);
+  // element j of the window sits at win[shift(k) + j], shift chosen so that shared and
+  // global addresses agree mod 16 B
+  auto shift_of = [&](int k) { return (int)(((xe + cb + (int64_t)(k - fip) * W) % 4 + 4) % 4); };
 
   // ---- prologue ---------------------------------------------------------------------
   for (int k = t; k <= KS; k += NTH) {
@@ -177,8 +183,8 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   const int rows = (int)min((int64_t)a.R, a.m - row0);
-  {  // acc := the far part's result for the panel rows (its slices combined in order, Q11);
-     // batches of 8 rows per thread, all loads in flight before the first use
+  {  // acc := the far part's result for the panel rows (its slices combined in order, Q11;
+     // none with P7); batches of 8 rows per thread, all loads in flight before the first use
     const VT* in = static_cast<const VT*>(a.init) + row0;
     for (int r0 = t; r0 < R; r0 += 8 * NTH) {
       double s[8];
@@ -204,27 +210,31 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     while (k < KS && sh.sp[k] == sh.sp[k + 1]) ++k;
     return k;
   };
-  auto issue = [&](int o) { issue_window<VT>(sh, bufs, L.bufbytes, x, a.n, xe, cb, W, KS, o); };
+  auto issue = [&](int ow) { issue_window<VT>(sh, bufs, L.bufbytes, x, a.n, xe, cb, W, KS, fip, ow); };
+  const int hf = fip && sh.sp[0] != sh.sp[1];  // the panel has a non-empty far slice (P7)
 
   const int64_t pb0 = a.panel_blk0[p];
   const int64_t tile0 = pb0 / PANEL_TC;  // first tile of the panel
+  // col16 holds band blocks only, far_col far-slice blocks only (P7)
+  const int64_t c16_off = fip ? a.far_blk0[p + 1] / PANEL_TC : 0;
   const uint64_t pol = pol_evict_first();
   const uint8_t* vbase = static_cast<const uint8_t*>(a.val);
   const uint8_t* cbase = static_cast<const uint8_t*>(a.col16);
   constexpr int VCH = BT * (int)sizeof(VT) / 16;  // 16-B chunks of values per thread
   constexpr int CCH = BT * 2 / 16;                 // 16-B chunks of u16 columns per thread
-  // this warp's tiles: in each non-empty slice, the slice's tiles wid, wid + NWARP, ...
-  int k = next_nonempty(0);
-  int o = 0;  // non-empty ordinal of slice k
+  constexpr int FCH = BT * 4 / 16;                 // 16-B chunks of int32 far columns per thread
 
   double ssq = 0.0;
+  int o = 0;  // non-empty ordinal of the current slice (the far slice included)
 
   // Warp NWARP-1 is the window producer; warps 0..NWARP-2 compute.  Between slices every
   // acc[row] must receive its slice o-1 sum before its slice o sum, and slice o-1's window
-  // buffer may take slice o+1 only when no warp reads it any more: named barrier X_o
-  // (bar.sync 1 + (o & 1), all NTH threads).  A compute warp that is done with slice o-1
+  // buffer may take a later band slice only when no warp reads it any more: named barrier
+  // X_o (barrier.sync 1 + (o & 1), all NTH threads; the non-.aligned form: a warp may
+  // arrive diverged after its lane-0 look-back or window requests).  A compute warp that is done with slice o-1
   // loads, multiplies and scans its first slice-o tile, and waits on X_o only before that
-  // tile's first acc update; the producer passes X_o and requests window o+1.
+  // tile's first acc update; the producer passes X_o and requests the next window.  With P7
+  // the far slice is slice 0 (no window; band window ordinal = o - hf).
   constexpr int NCW = NWARP - 1;
   if (wid == NWARP - 1) {
     int nne = 0;
@@ -234,22 +244,157 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       issue(1);
     }
     for (int oo = 1; oo < nne; ++oo) {
-      if (oo & 1) asm volatile("bar.sync 2, %0;" ::"n"(NTH) : "memory");
-      else asm volatile("bar.sync 1, %0;" ::"n"(NTH) : "memory");
-      if (lane == 0) issue(oo + 1);
+      if (oo & 1) asm volatile("barrier.sync 2, %0;" ::"n"(NTH) : "memory");
+      else asm volatile("barrier.sync 1, %0;" ::"n"(NTH) : "memory");
+      if (lane == 0 && oo - 1 >= hf) issue(oo + 1 - hf);  // slice oo-1 held window oo-1-hf
     }
-    k = KS;  // no tiles for the producer
   }
   auto slice_barrier = [&](int oo) {
-    if (oo & 1) asm volatile("bar.sync 2, %0;" ::"n"(NTH) : "memory");
-    else asm volatile("bar.sync 1, %0;" ::"n"(NTH) : "memory");
+    if (oo & 1) asm volatile("barrier.sync 2, %0;" ::"n"(NTH) : "memory");
+    else asm volatile("barrier.sync 1, %0;" ::"n"(NTH) : "memory");
   };
+
+  // ---- one tile after its products: per-thread segmented sum, warp scan, carry record,
+  // acc updates, look-back (shared by the far slice and the band slices) -----------------
+  auto finish = [&](VT(&pr)[BT], const uint32_t fl_, const int tr, const int lt, const int u, const int frk,
+                    bool& pending, auto&& prefetch) {
+    const uint32_t stops = ~fl_ & 0xFFFFu;
+    // per-thread segmented sum: pr[i] := sum of its segment up to block i
+    const int nst = __popc(stops);
+#pragma unroll
+    for (int i = 1; i < BT; ++i) pr[i] = ((stops >> (i - 1)) & 1u) ? pr[i] : pr[i - 1] + pr[i];
+    const VT tail = ((stops >> (BT - 1)) & 1u) ? VT(0) : pr[BT - 1];
+    // warp segmented scan of (has_stop, last partial sum); the stop count rides in
+    // the low 16 bits and the has-stop flag above (a sum of flags is non-zero iff their OR is)
+    int fn_ = nst | ((nst > 0) << 16);
+    VT v = tail;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
+      const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
+      if (lane >= d) {
+        if (!(fn_ >> 16)) v = v2 + v;
+        fn_ += g2;
+      }
+    }
+    const int f = (fn_ >> 16) != 0;
+    prefetch();  // the warp's next tile in flight during this tile's updates and look-back
+    // publish the tile's carry record (before anything waits on others); its carry-out is
+    // final at once when it holds a stop or starts its slice
+    const bool final_now = f || u == 0;
+    if (lane == 31) {
+      sh.rT[lt % RING] = v;  // inclusive: the tail after the tile's last stop, or its sum
+      if (final_now) sh.rI[lt % RING] = v;
+      __threadfence_block();
+      sh.rtag[lt % RING] = 2 * (lt + 1) + (final_now ? 1 : 0);
+    }
+    const int gx = __shfl_up_sync(0xffffffffu, fn_, 1);
+    int fx = (gx >> 16) != 0;
+    int nx = gx & 0xFFFF;
+    VT vx = __shfl_up_sync(0xffffffffu, v, 1);
+    if (lane == 0) {
+      fx = 0;
+      nx = 0;
+      vx = VT(0);
+    }
+    if (pending) {  // every warp is done with slice o - 1 (acc order)
+      slice_barrier(o);
+      pending = false;
+    }
+    // add the segment sums to acc[row]: the s-th stop of the slice is row first_row + s
+    // (reading P6), so this thread's stops take the rows from first_row + tile_rank + nx
+    // on.  The first stop also gets the earlier lanes' part (vx); when it continues earlier
+    // tiles (dep) their carry is added below, after the look-back — a fixed association,
+    // so y stays bitwise deterministic
+    const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
+    const int row_first = frk + tr + nx;
+    {
+      VT* ar = acc + row_first;
+      VT add = vx;
+#pragma unroll
+      for (int i = 0; i < BT; ++i)
+        if ((stops >> i) & 1u) {
+          *ar = *ar + (pr[i] + add);
+          add = VT(0);
+          ++ar;
+        }
+    }
+    // carry-in of the tile's first segment: decoupled look-back over the slice's earlier
+    // tiles back to the nearest one whose carry-out is final, then summed
+    // forward — the same left-to-right sum from the segment's start whichever record the
+    // walk stops at, so y is bitwise deterministic.  Needed by the warp's first stop (dep)
+    // and, for a tile without a stop, by its own carry-out (a row spanning many tiles walks
+    // O(warps) records per tile, not O(its length))
+    const bool nostop = !__shfl_sync(0xffffffffu, f, 31);
+    const unsigned dball = __ballot_sync(0xffffffffu, dep);
+    if (dball || (nostop && u > 0)) {
+      VT carry = VT(0);
+      if (lane == 0) {
+        int q = lt - 1;
+        for (;; --q) {
+          int tg;
+          while ((tg = sh.rtag[q % RING]) < 2 * (q + 1)) __nanosleep(16);
+          if (tg & 1) break;
+        }
+        __threadfence_block();
+        carry = sh.rI[q % RING];
+        for (int r = q + 1; r < lt; ++r) carry = carry + sh.rT[r % RING];
+      }
+      carry = __shfl_sync(0xffffffffu, carry, 0);
+      if (dep) acc[swz(row_first)] = acc[swz(row_first)] + carry;
+      if (nostop && lane == 31) {  // v of lane 31 = the tile's whole sum
+        sh.rI[lt % RING] = carry + v;
+        __threadfence_block();
+        sh.rtag[lt % RING] = 2 * (lt + 1) + 1;
+      }
+    }
+  };
+  // flow control (slices of more than LAG tiles only): the record slot of this tile must
+  // have been released — the tile LAG before it has a final carry-out
+  auto flow = [&](int lt, int u, int ntile_k) {
+    if (ntile_k > LAG && u >= LAG) {
+      if (lane == 0)
+        while (sh.rtag[(lt - LAG) % RING] != 2 * (lt - LAG + 1) + 1) __nanosleep(32);
+      __syncwarp();
+    }
+  };
+
+  // ---- P7: the far slice (slice 0): int32 columns, gathers of x from global memory -------
+  if (hf && wid < NCW) {
+    const int ntile_f = sh.sp[1] >> 9;
+    const int frk = sh.fr[0];
+    const int64_t ft0 = a.far_blk0[p] / PANEL_TC;  // the panel's first far-slice tile
+    const uint8_t* fcbase = static_cast<const uint8_t*>(a.far_col);
+    bool pending = false;
+    for (int u = wid; u < ntile_f; u += NCW) {
+      flow(u, u, ntile_f);
+      const int64_t tile = tile0 + u, ftile = ft0 + u;
+      uint32_t fc[BT], fv[VCH * 4];
+#pragma unroll
+      for (int c = 0; c < FCH; ++c)
+        ld16(fcbase + (ftile * (int64_t)32 * FCH + (int64_t)c * 32 + lane) * 16, pol, &fc[4 * c]);
+#pragma unroll
+      for (int c = 0; c < VCH; ++c)
+        ld16(vbase + (tile * (int64_t)32 * VCH + (int64_t)c * 32 + lane) * 16, pol, &fv[4 * c]);
+      const uint32_t flf = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
+      const int trf = __ldg(a.tile_rank + tile);
+      VT pr[BT];
+#pragma unroll
+      for (int i = 0; i < BT; ++i)  // column n: a FILLER block, reads 0 (P7)
+        pr[i] = fc[i] < (uint32_t)a.n ? __uint_as_float(fv[i]) * __ldg(x + fc[i]) : VT(0);
+      finish(pr, flf, trf, u, u, frk, pending, [] {});
+    }
+  }
+
+  // ---- the band slices -------------------------------------------------------------------
+  int k = wid < NCW ? next_nonempty(fip) : KS;  // no band tiles for the producer
+  o = hf;
   uint32_t vw[VCH * 4], cw[CCH * 4], fl = 0;
   int trank = 0;
   auto load_tile = [&](int lt) {  // panel-local tile: the thread's run (device layout)
-    const int64_t tile = tile0 + lt;
+    const int64_t tile = tile0 + lt, ctile = tile - c16_off;
 #pragma unroll
-    for (int c = 0; c < CCH; ++c) ld16(cbase + (tile * (int64_t)32 * CCH + (int64_t)c * 32 + lane) * 16, pol, &cw[4 * c]);
+    for (int c = 0; c < CCH; ++c) ld16(cbase + (ctile * (int64_t)32 * CCH + (int64_t)c * 32 + lane) * 16, pol, &cw[4 * c]);
 #pragma unroll
     for (int c = 0; c < VCH; ++c) ld16(vbase + (tile * (int64_t)32 * VCH + (int64_t)c * 32 + lane) * 16, pol, &vw[4 * c]);
     fl = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
@@ -265,31 +410,25 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     }
     return make_int2(kk, u);
   };
-  if (wid < NCW) {  // the warp's first tile in flight before the first window wait
+  if (k < KS) {  // the warp's first band tile in flight before the first window wait
     const int2 f = next_tile(k, wid - NCW);
     if (f.x < KS) load_tile((sh.sp[f.x] >> 9) + f.y);
   }
   while (k < KS) {
     const int ltile_k = sh.sp[k] >> 9;                     // panel-local first tile of the slice
     const int ntile_k = (sh.sp[k + 1] - sh.sp[k]) >> 9;    // tiles of the slice
-    // window o of slice k resident (a buffer two requests behind would alias the awaited
+    const int ow = o - hf;                                 // its window ordinal
+    // window ow of slice k resident (a buffer two requests behind would alias the awaited
     // parity: wait until the request is armed first)
-    while (sh.armed[o % PANEL_NBUF] != o) {
+    while (sh.armed[ow % PANEL_NBUF] != ow) {
     }
-    mbar_wait(&sh.bar[o % PANEL_NBUF], (o / PANEL_NBUF) & 1);
-    const VT* wk = win(o) + shift_of(k);
+    mbar_wait(&sh.bar[ow % PANEL_NBUF], (ow / PANEL_NBUF) & 1);
+    const VT* wk = win(ow) + shift_of(k);
     const int frk = sh.fr[k];
     bool pending = o > 0;  // X_o still ahead of this warp
     for (int u = wid; u < ntile_k; u += NCW) {
       const int lt = ltile_k + u;       // panel-local tile index (tag of its carry record)
-      // flow control (slices of more than LAG tiles only): the record slot of this tile
-      // must have been released
-      if (ntile_k > LAG && u >= LAG) {
-        if (lane == 0)
-          while (sh.rtag[(lt - LAG) % RING] != lt - LAG + 1) __nanosleep(32);
-        __syncwarp();
-      }
-
+      flow(lt, u, ntile_k);
       // ---- multiply: gathers from the slice's window --------------------------------
       VT pr[BT];
 #pragma unroll
@@ -297,86 +436,12 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
         const int c = (int)((cw[i >> 1] >> (16 * (i & 1))) & 0xFFFFu);
         pr[i] = __uint_as_float(vw[i]) * wk[c];
       }
-      const uint32_t stops = ~fl & 0xFFFFu;
-      const int tr = trank;
-      // ---- per-thread segmented sum: pr[i] := sum of its segment up to block i
-      const int nst = __popc(stops);
-#pragma unroll
-      for (int i = 1; i < BT; ++i) pr[i] = ((stops >> (i - 1)) & 1u) ? pr[i] : pr[i - 1] + pr[i];
-      const VT tail = ((stops >> (BT - 1)) & 1u) ? VT(0) : pr[BT - 1];
-      // ---- warp segmented scan of (has_stop, last partial sum); the stop count
-      // rides in the low 16 bits and the has-stop flag above (a sum of flags is non-zero
-      // iff their OR is) -----------------------------------------------------------------
-      int fn_ = nst | ((nst > 0) << 16);
-      VT v = tail;
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
-        const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
-        if (lane >= d) {
-          if (!(fn_ >> 16)) v = v2 + v;
-          fn_ += g2;
-        }
-      }
-      const int f = (fn_ >> 16) != 0;
-      {  // the warp's next tile in flight during this tile's updates and look-back
+      const uint32_t flc = fl;
+      const int trc = trank;
+      finish(pr, flc, trc, lt, u, frk, pending, [&] {
         const int2 nx2 = next_tile(k, u);
         if (nx2.x < KS) load_tile((sh.sp[nx2.x] >> 9) + nx2.y);
-      }
-      // ---- publish the tile's carry record (before anything waits on others) ----------
-      if (lane == 31) {
-        sh.rT[lt % RING] = v;   // inclusive: the tail after the tile's last stop, or its sum
-        sh.rH[lt % RING] = f;
-        __threadfence_block();
-        sh.rtag[lt % RING] = lt + 1;
-      }
-      const int gx = __shfl_up_sync(0xffffffffu, fn_, 1);
-      int fx = (gx >> 16) != 0;
-      int nx = gx & 0xFFFF;
-      VT vx = __shfl_up_sync(0xffffffffu, v, 1);
-      if (lane == 0) {
-        fx = 0;
-        nx = 0;
-        vx = VT(0);
-      }
-      if (pending) {  // every warp is done with slice o - 1 (acc order)
-        slice_barrier(o);
-        pending = false;
-      }
-      // ---- add the segment sums to acc[row]: the s-th stop of the slice is row
-      // first_row + s (reading P6), so this thread's stops take the rows from
-      // first_row + tile_rank + nx on.  The first stop also gets the earlier lanes' part
-      // (vx); when it continues earlier tiles (dep) their carry is added below, after the
-      // look-back — a fixed association, so y stays bitwise deterministic
-      const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
-      const int row_first = frk + tr + nx;
-      {
-        VT* ar = acc + row_first;
-        VT add = vx;
-#pragma unroll
-        for (int i = 0; i < BT; ++i)
-          if ((stops >> i) & 1u) {
-            *ar = *ar + (pr[i] + add);
-            add = VT(0);
-            ++ar;
-          }
-      }
-      // ---- carry-in of the first segment: decoupled look-back over the slice's earlier
-      // tiles (fold newest first back to the nearest tile holding a row stop)
-      const unsigned dball = __ballot_sync(0xffffffffu, dep);
-      if (dball) {
-        VT carry = VT(0);
-        if (lane == 0) {
-          for (int q = lt - 1; q >= ltile_k; --q) {
-            while (sh.rtag[q % RING] != q + 1) __nanosleep(16);
-            __threadfence_block();
-            carry = sh.rT[q % RING] + carry;
-            if (sh.rH[q % RING]) break;
-          }
-        }
-        carry = __shfl_sync(0xffffffffu, carry, 0);
-        if (dep) acc[swz(row_first)] = acc[swz(row_first)] + carry;
-      }
+      });
     }
     if (pending) slice_barrier(o);  // no tile of this slice: still part of X_o
     k = next_nonempty(k + 1);

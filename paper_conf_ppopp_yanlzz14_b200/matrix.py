@@ -38,7 +38,7 @@ def make_params(**kw) -> _lib.Params:
     p = _lib.Params()
     names = {"h": "block_h", "w": "block_w", "S": "slices", "T": "thread_tile", "C": "cta_size",
              "rc": "result_cache", "tpc": "tiles_per_cta", "B": "band", "R": "panel_rows", "W": "slice_width",
-             "col0": "band_col0"}
+             "col0": "band_col0", "far": "band_far"}
     for k, v in kw.items():
         setattr(p, names.get(k, k), int(v))
     return p
@@ -174,7 +174,8 @@ class Matrix:
     _ARR_DT = {"flags": np.uint8, "col_delta": np.int16, "seg_row": np.int32, "zero_rows": np.int32,
                "cta_seg0": np.int32, "fre": np.int32, "band_flags": np.uint8, "band_col16": np.uint16,
                "band_panel_blk0": np.int64, "band_slice_ptr": np.int32, "band_stop_ptr": np.int32,
-               "band_first_row": np.int32, "band_tile_rank": np.int32}
+               "band_first_row": np.int32, "band_tile_rank": np.int32, "band_far_col": np.int32,
+               "band_far_blk0": np.int64}
 
     def _arr_dtype(self, name: str):
         if name.startswith("val") or name == "band_val":

@@ -1,5 +1,5 @@
 """C5 at its full size (50M x 50M, ~1.0B non-zeros) in the launch configuration bench.py
-times (1x1, T=32, C=128, i32 columns, GPU translation): outputs the oracle can compute row
+times (bench.DEFAULT_PARAMS["c5"]): outputs the oracle can compute row
 by row are checked — a uniform sample of rows plus every long 'net' row (2^16-2^21 entries,
 spanning up to ~500 workgroup tiles, so their carries cross hundreds of CTAs) — for both
 the plain SpMV and the fused power-iteration step, plus run-to-run bitwise determinism."""
@@ -90,18 +90,21 @@ def test_c5_encoding_windows_bit_exact(c5):
     R, W, B = prm["panel_rows"], prm["slice_width"], prm["band"]
     S, T, C = prm["slices"], prm["thread_tile"], prm["cta_size"]
     assert B > 0 and info["band_panels"] == -(-csr.m // R)
+    fip = prm["band_far"] == 2
     blk0 = A.export("band_panel_blk0", device=True)
+    fblk0 = A.export("band_far_blk0", device=True) if fip else np.zeros_like(blk0)
     sptr = A.export("band_slice_ptr", device=True).reshape(info["band_panels"], -1)
     frow = A.export("band_first_row", device=True).reshape(info["band_panels"], -1)
-    far_flags = np.unpackbits(A.export("flags", device=True), bitorder="little")
-    far_stop = np.flatnonzero(far_flags[: info["nnzb"]] == 0)      # FILLER: stop k ends stacked row k
-    assert prm["empty_mode"] == E.EMPTY_FILLER and far_stop.size == S * csr.m
+    if not fip:
+        far_flags = np.unpackbits(A.export("flags", device=True), bitorder="little")
+        far_stop = np.flatnonzero(far_flags[: info["nnzb"]] == 0)      # FILLER: stop k ends stacked row k
+        assert prm["empty_mode"] == E.EMPTY_FILLER and far_stop.size == S * csr.m
     TCf = T * C
     for p0, p1 in _panel_windows(csr, R):
         r0, r1 = p0 * R, min(csr.m, p1 * R)
         sub = csr.row_slice(r0, r1)
         pp = PN.PanelParams(R=R, W=W, B=B, T=16, C=32, diag0=r0,
-                            far=E.Params(1, 1, S, T, C, prm["col_mode"], E.EMPTY_FILLER))
+                            far=E.Params(1, 1, S, T, C, prm["col_mode"], E.EMPTY_FILLER), far_in_panel=fip)
         # the window's slices use the full matrix' slice width of the far part
         enc = PN.encode_panel(sub.m, csr.n, sub.row_ptr, sub.col, sub.val, pp)
         # band stream: panels are independent, so the window's arrays are a slice of the whole
@@ -109,9 +112,15 @@ def test_c5_encoding_windows_bit_exact(c5):
         t0, nt = int(blk0[p0]) // 512, (int(blk0[p1]) - int(blk0[p0])) // 512
         assert nt == enc.nband_pad // 512
         assert np.array_equal(A.export_range("band_flags", t0, nt), enc.flags)
-        assert np.array_equal(A.export_range("band_col16", t0, nt), enc.col16)
         assert np.array_equal(A.export_range("band_val", t0, nt).view(np.uint32), enc.val.view(np.uint32))
         assert np.array_equal(A.export_range("band_tile_rank", t0, nt), enc.tile_rank)
+        # col16 counts band blocks only, far_col far-slice blocks only (P7)
+        f0, f1 = int(fblk0[p0]) // 512, int(fblk0[p1]) // 512
+        assert np.array_equal(A.export_range("band_col16", t0 - f0, nt - (f1 - f0)), enc.col16)
+        if fip:
+            assert np.array_equal(A.export_range("band_far_col", f0, f1 - f0), enc.far_col)
+            assert np.array_equal(fblk0[p0:p1 + 1] - fblk0[p0], enc.far_blk0)
+            continue
         # far part (BCCOO+, S slices stacked top-down): stacked rows s*m + [r0, r1)
         ef = enc.far
         ebits = np.unpackbits(ef.flags, bitorder="little")[: ef.nnzb]

@@ -1,4 +1,5 @@
-"""Panel-sliced BCCOO+ on the GPU (K4 panel_kernel after the far part's K1; DESIGN.md §2.1,
+"""Panel-sliced BCCOO+ on the GPU (K4 panel_kernel, with the far entries as a separate far
+part run by K1 first (the default) or as every panel's slice 0 (reading P7); DESIGN.md §2.1,
 §6.6) against the oracle: y = A x within the BASELINE.json tolerance per row (O1), bitwise
 exact with integer data, run-to-run deterministic; the uploaded band arrays read back from
 the device equal oracle/panel.py; the power-iteration epilogue; shapes that exercise the
@@ -62,14 +63,29 @@ CASES = {
     # far part as BCCOO+ (S = 2): its slice results are combined by the band kernel
     "c5-scaled-far-S2": (lambda: synth.circuit_like_rows(0, 400_000, n=400_000, band=8192, n_net=4,
                                                          net_log2=(12, 16)),
-                         dict(B=8192, R=4096, W=1024, S=2, T=32, C=128, col_mode=E.COL_I32)),
-    "webbase-far-S3": (lambda: synth.webbase_like(m=200_000), dict(B=1024, R=4096, W=512, S=3)),
+                         dict(B=8192, R=4096, W=1024, S=2, T=32, C=128, col_mode=E.COL_I32, far=1)),
+    "webbase-far-S3": (lambda: synth.webbase_like(m=200_000), dict(B=1024, R=4096, W=512, S=3, far=1)),
+    # P7: one far row of 2^17-2^18 entries per panel region (its far slice spans 256-512
+    # tiles: the look-back runs through tiles without a row stop) and panels whose far
+    # slices hold FILLER rows
+    "fip-long-rows": (lambda: synth.circuit_like_rows(0, 300_000, n=300_000, band=2000, n_net=3, net_log2=(16, 18),
+                                                      p_local=0.5),
+                      dict(B=2000, R=2048, W=1024, far=2)),
 }
+FARS = {"sep": 1, "fip": 2}
 
 
-@pytest.mark.parametrize("name", sorted(CASES))
-def test_tolerance_and_determinism(name):
+def _params(name, far):
     mk, params = CASES[name]
+    return mk, dict(params, far=params.get("far", FARS[far]))
+
+
+@pytest.mark.parametrize("far", sorted(FARS))
+@pytest.mark.parametrize("name", sorted(CASES))
+def test_tolerance_and_determinism(name, far):
+    if "far" in CASES[name][1] and CASES[name][1]["far"] != FARS[far]:
+        pytest.skip("the case fixes its far mode")
+    mk, params = _params(name, far)
     csr = mk()
     x = synth.make_x(csr.n, np.float32, "uniform", 1)
     A = _build(csr, **params)
@@ -85,9 +101,10 @@ def test_tolerance_and_determinism(name):
         A.free()
 
 
-@pytest.mark.parametrize("name", ["c5-scaled", "small-many-slices", "col0-neg", "tiny-m", "c5-scaled-far-S2"])
-def test_integer_exact(name):
-    mk, params = CASES[name]
+@pytest.mark.parametrize("far", sorted(FARS))
+@pytest.mark.parametrize("name", ["c5-scaled", "small-many-slices", "col0-neg", "tiny-m", "fip-long-rows"])
+def test_integer_exact(name, far):
+    mk, params = _params(name, far)
     csr0 = mk()
     csr = synth.CSR(csr0.m, csr0.n, csr0.row_ptr, csr0.col,
                     np.random.default_rng(3).integers(-3, 4, csr0.nnz).astype(np.float32))
@@ -101,15 +118,17 @@ def test_integer_exact(name):
         A.free()
 
 
-@pytest.mark.parametrize("name", ["c5-scaled", "col0-pos", "small-many-slices"])
-def test_device_arrays_equal_oracle(name):
-    mk, params = CASES[name]
+@pytest.mark.parametrize("far", sorted(FARS))
+@pytest.mark.parametrize("name", ["c5-scaled", "col0-pos", "small-many-slices", "fip-long-rows"])
+def test_device_arrays_equal_oracle(name, far):
+    mk, params = _params(name, far)
     csr = mk()
     from paper_conf_ppopp_yanlzz14_b200._lib import PANEL_BC, PANEL_BT
-    far = E.Params(1, 1, 1, params.get("T", 16), params.get("C", 256), params.get("col_mode", 0),
-                   params.get("empty_mode", 0))
+    farp = E.Params(1, 1, 1, params.get("T", 16), params.get("C", 256), params.get("col_mode", 0),
+                    params.get("empty_mode", 0))
+    fip = params["far"] == 2
     pp = PN.PanelParams(R=params.get("R", 16384), W=params.get("W", 16384), B=params["B"], T=PANEL_BT, C=PANEL_BC,
-                        diag0=params.get("col0", 0), far=far)
+                        diag0=params.get("col0", 0), far=farp, far_in_panel=fip)
     enc = PN.encode_panel(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, pp)
     A = _build(csr, **params)
     try:
@@ -120,8 +139,12 @@ def test_device_arrays_equal_oracle(name):
         assert np.array_equal(A.export("band_tile_rank", device=True), enc.tile_rank)
         assert np.array_equal(A.export("band_slice_ptr", device=True), enc.slice_ptr.ravel())
         assert np.array_equal(A.export("band_stop_ptr", device=True), enc.stop_ptr.ravel())
-        assert np.array_equal(A.export("flags", device=True), enc.far.flags)
-        assert np.array_equal(A.export("col", device=True), enc.far.col)
+        if fip:
+            assert np.array_equal(A.export("band_far_col", device=True), enc.far_col)
+            assert np.array_equal(A.export("band_far_blk0", device=True), enc.far_blk0)
+        else:
+            assert np.array_equal(A.export("flags", device=True), enc.far.flags)
+            assert np.array_equal(A.export("col", device=True), enc.far.col)
     finally:
         A.free()
 
@@ -138,9 +161,10 @@ def test_gpu_encoded_far_part():
         A.free()
 
 
-@pytest.mark.parametrize("name", ["c5-scaled", "webbase", "webbase-far-S3"])
-def test_power_step(name):
-    mk, params = CASES[name]
+@pytest.mark.parametrize("name,far", [("c5-scaled", "sep"), ("c5-scaled", "fip"), ("webbase", "fip"),
+                                      ("webbase-far-S3", "sep")])
+def test_power_step(name, far):
+    mk, params = _params(name, far)
     csr0 = mk()
     csr = synth.CSR(csr0.m, csr0.n, csr0.row_ptr, csr0.col,
                     np.random.default_rng(4).integers(-2, 3, csr0.nnz).astype(np.float32))
@@ -156,7 +180,7 @@ def test_power_step(name):
         torch.cuda.synchronize()
         assert np.array_equal(y.cpu().numpy().astype(np.float64), ye / 2)
         assert out.item() == float(np.sum((ye / 2) ** 2))
-        assert A.launches_per_spmv() == 2
+        assert A.launches_per_spmv() == (1 if params["far"] == 2 else 2)
     finally:
         A.free()
 
@@ -173,8 +197,9 @@ def test_host_buffers():
 
 
 def test_tune_and_reencode_keep_the_band():
-    """yaspmv_tune on a panel-sliced handle tunes its far part (Table 1 over 1x1 blocks) and
-    keeps the band stream; yaspmv_reencode(band = -1) returns to the plain format."""
+    """yaspmv_tune on a panel-sliced handle times the far entries inside the panels (P7)
+    against a separate far part tuned over Table 1 (1x1 blocks) and keeps the band stream;
+    yaspmv_reencode(band = -1) returns to the plain format."""
     mk, params = CASES["webbase"]
     csr = mk()
     x = synth.make_x(csr.n, np.float32, "uniform", 7)
@@ -183,7 +208,8 @@ def test_tune_and_reencode_keep_the_band():
         chosen = A.tune()
         info = A.info()
         assert info["band_blocks"] > 0 and chosen["block_h"] == chosen["block_w"] == 1
-        assert info["params"]["band"] == params["B"]
+        assert info["params"]["band"] == params["B"] and chosen["band_far"] in (1, 2)
+        assert info["params"]["band_far"] == chosen["band_far"]
         _check(csr, _run(A, x), x)
         A.reencode(B=-1)
         assert A.info()["band_blocks"] == 0
