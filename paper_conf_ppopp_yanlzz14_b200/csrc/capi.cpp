@@ -11,6 +11,7 @@
 #include <cstdlib>
 
 #include "handle.hpp"
+#include "trace.hpp"
 #include "../../include/yaspmv_ablation.h"
 
 using namespace yaspmv;
@@ -737,6 +738,7 @@ const char* yaspmv_version(void) { return "yaspmv-b200 0.1 (sm_100a)"; }
 yaspmv_status yaspmv_build_csr(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                                const void* vals, yaspmv_dtype dtype, const yaspmv_params* params,
                                int32_t device, yaspmv_matrix* out) {
+  yaspmv::TraceRange tr_("yaspmv:build_csr");
   if (!out) return fail(YASPMV_EINVAL, "out is NULL");
   *out = nullptr;
   if (dtype != YASPMV_F32 && dtype != YASPMV_F64) return fail(YASPMV_EINVAL, "bad dtype");
@@ -756,6 +758,7 @@ yaspmv_status yaspmv_build_csr(int64_t m, int64_t n, const int64_t* row_ptr, con
 yaspmv_status yaspmv_build_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row_idx, const int32_t* col_idx,
                                const void* vals, yaspmv_dtype dtype, const yaspmv_params* params, int32_t device,
                                yaspmv_matrix* out) {
+  yaspmv::TraceRange tr_("yaspmv:build_coo");
   if (!out) return fail(YASPMV_EINVAL, "out is NULL");
   *out = nullptr;
   if (dtype != YASPMV_F32 && dtype != YASPMV_F64) return fail(YASPMV_EINVAL, "bad dtype");
@@ -810,6 +813,7 @@ yaspmv_status yaspmv_profile_end(yaspmv_matrix A, double* ms, int32_t n, int64_t
 }
 
 yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
+  yaspmv::TraceRange tr_("yaspmv:reencode");
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (!A->have_csr) return fail(YASPMV_EINVAL, "handle was built with YASPMV_DROP_CSR");
   Params want = from_abi(params);
@@ -847,6 +851,7 @@ yaspmv_status yaspmv_reencode(yaspmv_matrix A, const yaspmv_params* params) {
 }
 
 yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream) {
+  yaspmv::TraceRange tr_("yaspmv:spmv");
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle (built with device = -1): no CPU fallback");
   if (A->can.m > 0 && !y) return fail(YASPMV_EINVAL, "y is NULL");
@@ -862,6 +867,7 @@ yaspmv_status yaspmv_spmv(yaspmv_matrix A, const void* x, void* y, void* stream)
 
 yaspmv_status yaspmv_spmv_power(yaspmv_matrix A, const void* x, void* y, const double* in_norm2, double* out_norm2,
                                 void* stream) {
+  yaspmv::TraceRange tr_("yaspmv:spmv_power");
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle (built with device = -1): no CPU fallback");
   if (A->can.m > 0 && !y) return fail(YASPMV_EINVAL, "y is NULL");
@@ -876,6 +882,7 @@ yaspmv_status yaspmv_spmv_power(yaspmv_matrix A, const void* x, void* y, const d
 }
 
 yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host, void* stream) {
+  yaspmv::TraceRange tr_("yaspmv:spmv_host");
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle: no CPU fallback");
   const size_t xb = (size_t)A->can.n * A->vsize, yb = (size_t)A->can.m * A->vsize;
@@ -892,6 +899,7 @@ yaspmv_status yaspmv_spmv_host(yaspmv_matrix A, const void* x_host, void* y_host
 }
 
 yaspmv_status yaspmv_spmv_host_async(yaspmv_matrix A, const void* x_host, void* y_host, void* stream) {
+  yaspmv::TraceRange tr_("yaspmv:spmv_host_async");
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle: no CPU fallback");
   const size_t xb = (size_t)A->can.n * A->vsize, yb = (size_t)A->can.m * A->vsize;

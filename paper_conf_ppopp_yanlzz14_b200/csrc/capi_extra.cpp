@@ -10,6 +10,7 @@
 #include <vector>
 
 #include "handle.hpp"
+#include "trace.hpp"
 
 using namespace yaspmv;
 
@@ -263,6 +264,7 @@ yaspmv_status yaspmv_export_device_range(yaspmv_matrix A, int32_t which, int64_t
 
 // ------------------------------------------------------------------ auto-tuner (§4)
 yaspmv_status yaspmv_tune_ex(yaspmv_matrix A, void* stream, yaspmv_params* chosen, int32_t mode) {
+  yaspmv::TraceRange tr_("yaspmv:tune_ex");
   if (!A) return fail(YASPMV_EINVAL, "NULL handle");
   if (A->device < 0) return fail(YASPMV_EINVAL, "tuning times the kernels: needs a device handle");
   if (!A->have_csr) return fail(YASPMV_EINVAL, "handle was built with YASPMV_DROP_CSR");

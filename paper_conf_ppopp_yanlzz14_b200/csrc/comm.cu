@@ -20,6 +20,7 @@
 #include <string>
 
 #include "handle.hpp"
+#include "trace.hpp"
 
 using namespace yaspmv;
 
@@ -265,6 +266,7 @@ yaspmv_status yaspmv_comm_wait(yaspmv_comm c, void* stream) {
 }
 
 yaspmv_status yaspmv_power_step_fused(yaspmv_matrix A, yaspmv_comm c, void* stream) {
+  yaspmv::TraceRange tr_("yaspmv:power_step_fused");
   if (!A || !c) return fail(YASPMV_EINVAL, "NULL argument");
   if (A->device < 0) return fail(YASPMV_EINVAL, "host-only handle: no CPU fallback");
   if (!c->connected) return fail(YASPMV_EINVAL, "comm not connected (open_ipc / connect_local)");
