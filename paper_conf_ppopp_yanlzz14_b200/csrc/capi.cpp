@@ -687,6 +687,9 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   pa.KS = g.NS();
   pa.npanels = g.npanels;
   pa.epi = (in_norm2 ? 1 : 0) | (out_norm2 ? 2 : 0);
+  // the band kernel as a programmatic dependent of the far kernel just launched (not after
+  // a memset, not with P7, whose far phase gathers x at once)
+  pa.pdl = (!fip && A->can.ntiles > 0 && !(A->can.p.flags & YASPMV_NO_PDL)) ? 1 : 0;
   pa.in_norm2 = in_norm2;
   pa.part = A->pd.part;
   const int e = launch_panel(pa, A->dtype, stream);

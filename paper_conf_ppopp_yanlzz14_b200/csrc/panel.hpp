@@ -110,6 +110,7 @@ struct PanelArgs {
   int64_t m, n;
   int64_t R, W, B, col0, KS, npanels;
   int epi;            // bit 0: scale by 1/sqrt(*in_norm2); bit 1: part[p] = sum over the panel of y^2
+  int pdl;            // launched as a programmatic dependent of the far kernel (see launch_panel)
   const double* in_norm2;
   double* part;
 };

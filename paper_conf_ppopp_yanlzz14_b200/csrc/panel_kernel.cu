@@ -2,10 +2,9 @@
 // §6.6).  One CTA per row panel of R rows (PAPER.md's workgroup, walking the
 // panel's band stream in workgroup-level tiles of BT*BC blocks):
 //
-//   prologue  acc[0..R) := the far part's result (its S slice vectors summed in fp64), or
-//             0 when the far entries are the panel's slice 0 (reading P7); the panel's
-//             slice offsets to shared memory; the x windows of the first two band slices
-//             (W values each) requested with cp.async.bulk on an mbarrier — the part of x
+//   prologue  acc[0..R) := 0; the panel's slice offsets to shared memory; the x windows
+//             of the first two band slices (W values each) requested with cp.async.bulk
+//             on an mbarrier — the part of x
 //             one BCCOO+ slice uses, staged in shared memory so that every gather
 //             of the slice is an LDS instead of a 32-byte L2 request;
 //   P7        the far slice first: the same tiles with int32 columns, x gathered from
@@ -24,7 +23,8 @@
 //             from the tile's first-result entry (reading P6).  Inside a slice every row has one segment, so no
 //             two warps touch one row; a barrier between slices keeps each row's slice
 //             sums in ascending order (the BCCOO+ combine order) — deterministic;
-//   epilogue  y[panel rows] := acc (optionally scaled; per-panel sum of y^2).
+//   epilogue  y[panel rows] := the far part's result (its S slice vectors summed in fp64; none
+//             with P7) + acc, optionally scaled; per-panel sum of y^2.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -183,28 +183,9 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   const int rows = (int)min((int64_t)a.R, a.m - row0);
-  {  // acc := the far part's result for the panel rows (its slices combined in order, Q11;
-     // none with P7); batches of 8 rows per thread, all loads in flight before the first use
-    const VT* in = static_cast<const VT*>(a.init) + row0;
-    for (int r0 = t; r0 < R; r0 += 8 * NTH) {
-      double s[8];
-#pragma unroll
-      for (int j = 0; j < 8; ++j) s[j] = 0.0;
-      for (int q = 0; q < a.ninit; ++q) {
-        VT v[8];
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int r = r0 + j * NTH;
-          v[j] = r < rows ? __ldcs(in + q * a.init_stride + r) : VT(0);
-        }
-#pragma unroll
-        for (int j = 0; j < 8; ++j) s[j] += (double)v[j];
-      }
-#pragma unroll
-      for (int j = 0; j < 8; ++j)
-        if (r0 + j * NTH < R) acc[swz(r0 + j * NTH)] = (VT)s[j];
-    }
-  }
+  // acc := 0 (the far part's result joins in the epilogue, after this grid's wait on it)
+  for (int r = t * (16 / (int)sizeof(VT)); r < R; r += NTH * (16 / (int)sizeof(VT)))
+    *reinterpret_cast<uint4*>(acc + r) = make_uint4(0u, 0u, 0u, 0u);
   __syncthreads();
   auto next_nonempty = [&](int k) {  // first slice >= k holding blocks (KS: none)
     while (k < KS && sh.sp[k] == sh.sp[k + 1]) ++k;
@@ -247,6 +228,18 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       if (oo & 1) asm volatile("barrier.sync 2, %0;" ::"n"(NTH) : "memory");
       else asm volatile("barrier.sync 1, %0;" ::"n"(NTH) : "memory");
       if (lane == 0 && oo - 1 >= hf) issue(oo + 1 - hf);  // slice oo-1 held window oo-1-hf
+    }
+    // the far part's slice results of the panel rows, wanted by the epilogue: once the far
+    // kernel is complete (programmatic dependent launch), pulled into L2 in the background
+    if (a.ninit > 0 && rows > 0) {
+      if (a.pdl) cudaGridDependencySynchronize();
+      if (lane < a.ninit) {
+        const VT* in = static_cast<const VT*>(a.init) + row0 + lane * a.init_stride;
+        const uintptr_t b0 = reinterpret_cast<uintptr_t>(in) & ~(uintptr_t)15;
+        const uintptr_t b1 = reinterpret_cast<uintptr_t>(in + rows) & ~(uintptr_t)15;
+        if (b1 > b0)
+          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b0), "r"((unsigned)(b1 - b0)) : "memory");
+      }
     }
   }
   auto slice_barrier = [&](int oo) {
@@ -303,21 +296,20 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     }
     // add the segment sums to acc[row]: the s-th stop of the slice is row first_row + s
     // (reading P6), so this thread's stops take the rows from first_row + tile_rank + nx
-    // on.  The first stop also gets the earlier lanes' part (vx); when it continues earlier
-    // tiles (dep) their carry is added below, after the look-back — a fixed association,
-    // so y stays bitwise deterministic
+    // on.  The first stop's row then also gets the earlier lanes' part (vx) — right away,
+    // or, when the segment continues earlier tiles (dep), together with their carry after
+    // the look-back: a fixed association, so y stays bitwise deterministic
     const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
     const int row_first = frk + tr + nx;
     {
       VT* ar = acc + row_first;
-      VT add = vx;
 #pragma unroll
       for (int i = 0; i < BT; ++i)
         if ((stops >> i) & 1u) {
-          *ar = *ar + (pr[i] + add);
-          add = VT(0);
+          *ar = *ar + pr[i];
           ++ar;
         }
+      if (nst && !dep) acc[swz(row_first)] = acc[swz(row_first)] + vx;
     }
     // carry-in of the tile's first segment: decoupled look-back over the slice's earlier
     // tiles back to the nearest one whose carry-out is final, then summed
@@ -341,7 +333,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
         for (int r = q + 1; r < lt; ++r) carry = carry + sh.rT[r % RING];
       }
       carry = __shfl_sync(0xffffffffu, carry, 0);
-      if (dep) acc[swz(row_first)] = acc[swz(row_first)] + carry;
+      if (dep) acc[swz(row_first)] = acc[swz(row_first)] + (carry + vx);
       if (nostop && lane == 31) {  // v of lane 31 = the tile's whole sum
         sh.rI[lt % RING] = carry + v;
         __threadfence_block();
@@ -400,19 +392,16 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     fl = ld_flags16(a.flags + ((tile * PANEL_TC + (int64_t)lane * BT) >> 3));
     trank = __ldg(a.tile_rank + tile);
   };
-  // this warp's tile after (kk, u): the next one of the slice, else its first tile of the
-  // next non-empty slice that has one (kk = KS: none)
-  auto next_tile = [&](int kk, int u) {
-    u += NCW;
-    while (kk < KS && (sh.sp[kk + 1] - sh.sp[kk]) >> 9 <= u) {
-      kk = next_nonempty(kk + 1);
-      u = wid;
-    }
-    return make_int2(kk, u);
+  // this warp's first tile in slice kk or a later non-empty slice that has one: its
+  // panel-local tile index, -1 if none
+  auto first_tile_from = [&](int kk) {
+    kk = next_nonempty(kk);
+    while (kk < KS && (sh.sp[kk + 1] - sh.sp[kk]) >> 9 <= wid) kk = next_nonempty(kk + 1);
+    return kk < KS ? (sh.sp[kk] >> 9) + wid : -1;
   };
   if (k < KS) {  // the warp's first band tile in flight before the first window wait
-    const int2 f = next_tile(k, wid - NCW);
-    if (f.x < KS) load_tile((sh.sp[f.x] >> 9) + f.y);
+    const int f = first_tile_from(k);
+    if (f >= 0) load_tile(f);
   }
   while (k < KS) {
     const int ltile_k = sh.sp[k] >> 9;                     // panel-local first tile of the slice
@@ -438,9 +427,13 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       }
       const uint32_t flc = fl;
       const int trc = trank;
-      finish(pr, flc, trc, lt, u, frk, pending, [&] {
-        const int2 nx2 = next_tile(k, u);
-        if (nx2.x < KS) load_tile((sh.sp[nx2.x] >> 9) + nx2.y);
+      finish(pr, flc, trc, lt, u, frk, pending, [&] {  // the warp's next tile
+        if (u + NCW < ntile_k) {
+          load_tile(lt + NCW);
+        } else {
+          const int f = first_tile_from(k + 1);
+          if (f >= 0) load_tile(f);
+        }
       });
     }
     if (pending) slice_barrier(o);  // no tile of this slice: still part of X_o
@@ -449,12 +442,34 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   }
   __syncthreads();  // the last slice's sums are in acc
 
-  // ---- epilogue: y := acc (scaled), sum of y^2 ----------------------------------------
+  // ---- epilogue: y := far part + acc (scaled), sum of y^2 -------------------------------
+  // y[r] = (s_0 + ... + s_{S-1}) + band, the far part's S slice results summed in ascending
+  // order in fp64 (the BCCOO+ combine, Q11) and the band slices' fp32 sum added to it
+  // in fp64: a fixed association, bitwise deterministic
+  if (a.pdl && a.ninit > 0) cudaGridDependencySynchronize();  // the far kernel is complete
   const double inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
-  for (int r = t; r < rows; r += NTH) {
-    const VT o2 = (a.epi & 1) ? (VT)(acc[swz(r)] * inv) : acc[swz(r)];
-    y[row0 + r] = o2;
-    ssq += (double)o2 * (double)o2;
+  const VT* in = static_cast<const VT*>(a.init) + row0;
+  for (int r0 = t; r0 < rows; r0 += 4 * NTH) {
+    double s[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) s[j] = 0.0;
+    for (int q = 0; q < a.ninit; ++q) {
+      VT v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) v[j] = r0 + j * NTH < rows ? __ldcs(in + q * a.init_stride + r0 + j * NTH) : VT(0);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) s[j] += (double)v[j];
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int r = r0 + j * NTH;
+      if (r < rows) {
+        const VT o2 = a.ninit > 0 ? (VT)((s[j] + (double)acc[swz(r)]) * inv)
+                                  : ((a.epi & 1) ? (VT)(acc[swz(r)] * inv) : acc[swz(r)]);
+        y[row0 + r] = o2;
+        ssq += (double)o2 * (double)o2;
+      }
+    }
   }
   if (a.epi & 2) {
 #pragma unroll
@@ -496,8 +511,20 @@ int panel_attr(int64_t R, int64_t W, int* regs) {
 int launch_panel(const PanelArgs& a, int dtype, void* stream) {
   if (dtype != 0) return (int)cudaErrorNotSupported;
   if (a.npanels == 0) return 0;
-  panel_kernel<float><<<(unsigned)a.npanels, NTH, panel_smem_bytes(a.R, a.W), (cudaStream_t)stream>>>(a);
-  return (int)cudaGetLastError();
+  // programmatic dependent launch (a.pdl): the CTAs may start while the far kernel's last
+  // wave runs — that kernel lets dependents launch only after each of its CTAs has waited
+  // for its own predecessors, so x is final; its results are read after this grid waits
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)a.npanels);
+  cfg.blockDim = dim3(NTH);
+  cfg.dynamicSmemBytes = panel_smem_bytes(a.R, a.W);
+  cfg.stream = (cudaStream_t)stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return (int)cudaLaunchKernelEx(&cfg, panel_kernel<float>, a);
 }
 
 }  // namespace yaspmv

@@ -444,7 +444,13 @@ __device__ __forceinline__ void stream_tile(const KArgs& a, const int64_t tile, 
   // written by other kernels) and overlaps the previous kernel's tail; x, y, the status
   // words and the ticket may depend on earlier kernels in the stream.
   if (a.block_ids) {
-    if (a.pdl) cudaGridDependencySynchronize();
+    // the next kernel may launch once every CTA is past this wait: whatever it reads that
+    // an earlier kernel wrote (x) is then final (the panel kernel reads x before it waits
+    // for this grid's own results)
+    if (a.pdl) {
+      cudaGridDependencySynchronize();
+      cudaTriggerProgrammaticLaunchCompletion();
+    }
     if (t == 0) {
       tk = atomicAdd(a.ticket, 1ull);  // consumed only at the scan barrier (epoch)
       if constexpr (EPI == 1 || EPI == 2) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
@@ -915,7 +921,6 @@ template <typename VT, int H, int W, int T, int CM, int EPI>
 __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_kernel(const KArgs a) {
   __shared__ ScanShared<VT, H> shb[2];
   ScanShared<VT, H>& sh = shb[0];
-  if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();  // the next SpMV may start its loads
   if (a.block_ids) {  // tile = workgroup id: workgroups dispatch in order — the default
     if (a.tpc <= 1) {
       tile_body<VT, H, W, T, CM, EPI>(a, (int64_t)blockIdx.x, sh);
@@ -930,7 +935,10 @@ __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_kerne
     for (int64_t tile = t0; tile < t1; ++tile) tile_body<VT, H, W, T, CM, EPI>(a, tile, shb[tile & 1]);
     return;
   }
-  if (a.pdl) cudaGridDependencySynchronize();
+  if (a.pdl) {
+    cudaGridDependencySynchronize();
+    cudaTriggerProgrammaticLaunchCompletion();
+  }
   if (threadIdx.x == 0) {  // logical workgroup id from an atomic ticket
     const unsigned long long tk = atomicAdd(a.ticket, 1ull);
     const unsigned long long q = tk / (unsigned long long)a.period;
@@ -948,7 +956,6 @@ __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_s2_ke
   __shared__ ScanShared<VT, H> sh;
   extern __shared__ __align__(16) unsigned char s2_rcache[];
   VT* rcache = reinterpret_cast<VT*>(s2_rcache);
-  if (a.pdl) cudaTriggerProgrammaticLaunchCompletion();
   if (a.block_ids) {
     // consecutive tiles without a barrier in between: each state (counts, scan values,
     // result cache) is written in tile k+1 only after a barrier that every warp reaches
@@ -958,7 +965,10 @@ __global__ void __maxnreg__((KTraits<VT, H, W, T, CM>::MAXREG)) spmv_bccoo_s2_ke
     for (int64_t tile = t0; tile < t1; ++tile) tile_body_s2<VT, H, W, T, CM, EPI>(a, tile, sh, rcache);
     return;
   }
-  if (a.pdl) cudaGridDependencySynchronize();
+  if (a.pdl) {
+    cudaGridDependencySynchronize();
+    cudaTriggerProgrammaticLaunchCompletion();
+  }
   if (threadIdx.x == 0) {
     const unsigned long long tk = atomicAdd(a.ticket, 1ull);
     const unsigned long long q = tk / (unsigned long long)a.period;
