@@ -71,6 +71,7 @@ def main():
         for _ in range(3):
             call()
         ts = []
+        A.profile_begin()
         for _ in range(args.iters):
             if args.flush:
                 scratch.zero_()
@@ -78,12 +79,14 @@ def main():
             a.record(); call(); b.record()
             torch.cuda.synchronize()
             ts.append(a.elapsed_time(b))
+        prof = A.profile_end()
         info = A.info()
         ms = float(np.median(ts))
+        kern = {k: v / max(prof.get("calls", 1), 1) for k, v in prof.items() if k.endswith("_ms")}
         print(json.dumps({"params": {k: v for k, v in info["params"].items() if k != "flags"}, "ms": ms,
                           "min_ms": float(np.min(ts)), "alg_GBs": info["alg_bytes"] / ms / 1e6,
                           "gflops": 2 * info["nnz"] / ms / 1e6, "regs": info["regs_per_thread"],
-                          "alg_bytes": info["alg_bytes"], "build_s": tb}), flush=True)
+                          "alg_bytes": info["alg_bytes"], "build_s": tb, "kern_ms": kern}), flush=True)
         A.free()
 
 
