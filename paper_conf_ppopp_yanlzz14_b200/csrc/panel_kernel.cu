@@ -302,13 +302,26 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     const bool dep = nst && !fx && u > 0;  // the warp's first stop continues earlier tiles
     const int row_first = frk + tr + nx;
     {
-      VT* ar = acc + row_first;
+      // four independent update chains, one per quarter of the thread tile (positions
+      // 4q..4q+3 own the rows from row_first + the stops before 4q on): their loads issue
+      // back to back instead of one shared-memory round trip per stop; the chains touch
+      // disjoint rows, so the result is the same as the sequential walk
+      static_assert(BT == 16, "four chains of four positions");
+      const int c1 = __popc(stops & 0xFu), c2 = c1 + __popc(stops & 0xF0u), c3 = c2 + __popc(stops & 0xF00u);
+      VT* aq[4] = {acc + row_first, acc + row_first + c1, acc + row_first + c2, acc + row_first + c3};
 #pragma unroll
-      for (int i = 0; i < BT; ++i)
-        if ((stops >> i) & 1u) {
-          *ar = *ar + pr[i];
-          ++ar;
-        }
+      for (int r = 0; r < 4; ++r) {
+        VT l[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if ((stops >> (4 * q + r)) & 1u) l[q] = *aq[q];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if ((stops >> (4 * q + r)) & 1u) {
+            *aq[q] = l[q] + pr[4 * q + r];
+            ++aq[q];
+          }
+      }
       if (nst && !dep) acc[swz(row_first)] = acc[swz(row_first)] + vx;
     }
     // carry-in of the tile's first segment: decoupled look-back over the slice's earlier
@@ -449,27 +462,71 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   if (a.pdl && a.ninit > 0) cudaGridDependencySynchronize();  // the far kernel is complete
   const double inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   const VT* in = static_cast<const VT*>(a.init) + row0;
-  for (int r0 = t; r0 < rows; r0 += 4 * NTH) {
-    double s[4];
+  // y[r] = (VT)((s_0 + ... + s_{S-1} in fp64, ascending) + acc[r]) * inv)
+  auto out_row = [&](int r, double s) {
+    const VT o2 = a.ninit > 0 ? (VT)((s + (double)acc[swz(r)]) * inv)
+                              : ((a.epi & 1) ? (VT)(acc[swz(r)] * inv) : acc[swz(r)]);
+    y[row0 + r] = o2;
+    ssq += (double)o2 * (double)o2;
+  };
+  int rdone = 0;
+  if (sizeof(VT) == 4 && ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(y + row0)) & 15) == 0 &&
+      (a.init_stride & 3) == 0) {
+    // 128-bit loads of the far part's slice results, every slice of two row quads in flight
+    // at once (the epilogue runs with no other CTA on the SM to hide its latency)
+    const int ng = rows >> 2;
+    for (int g0 = t; g0 < ng; g0 += 2 * NTH) {
+      double s[2][4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) s[j] = 0.0;
-    for (int q = 0; q < a.ninit; ++q) {
-      VT v[4];
+      for (int h = 0; h < 2; ++h)
 #pragma unroll
-      for (int j = 0; j < 4; ++j) v[j] = r0 + j * NTH < rows ? __ldcs(in + q * a.init_stride + r0 + j * NTH) : VT(0);
+        for (int j = 0; j < 4; ++j) s[h][j] = 0.0;
+      for (int q0 = 0; q0 < a.ninit; q0 += 4) {
+        float4 v[4][2];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) s[j] += (double)v[j];
-    }
+        for (int dq = 0; dq < 4; ++dq)
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int r = r0 + j * NTH;
-      if (r < rows) {
-        const VT o2 = a.ninit > 0 ? (VT)((s[j] + (double)acc[swz(r)]) * inv)
-                                  : ((a.epi & 1) ? (VT)(acc[swz(r)] * inv) : acc[swz(r)]);
-        y[row0 + r] = o2;
-        ssq += (double)o2 * (double)o2;
+          for (int h = 0; h < 2; ++h) {
+            const int g = g0 + h * NTH;
+            v[dq][h] = (q0 + dq < a.ninit && g < ng)
+                           ? __ldcs(reinterpret_cast<const float4*>(in + (int64_t)(q0 + dq) * a.init_stride) + g)
+                           : make_float4(0.f, 0.f, 0.f, 0.f);
+          }
+#pragma unroll
+        for (int dq = 0; dq < 4; ++dq)
+          if (q0 + dq < a.ninit)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              s[h][0] += (double)v[dq][h].x;
+              s[h][1] += (double)v[dq][h].y;
+              s[h][2] += (double)v[dq][h].z;
+              s[h][3] += (double)v[dq][h].w;
+            }
+      }
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int g = g0 + h * NTH;
+        if (g < ng) {
+          const float4 ac = *reinterpret_cast<const float4*>(acc + 4 * g);
+          float4 o;
+          const float ai[4] = {ac.x, ac.y, ac.z, ac.w};
+          float oi[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            oi[j] = a.ninit > 0 ? (float)((s[h][j] + (double)ai[j]) * inv) : ((a.epi & 1) ? (float)(ai[j] * inv) : ai[j]);
+            ssq += (double)oi[j] * (double)oi[j];
+          }
+          o = make_float4(oi[0], oi[1], oi[2], oi[3]);
+          *reinterpret_cast<float4*>(y + row0 + 4 * g) = o;
+        }
       }
     }
+    rdone = ng * 4;
+  }
+  for (int r = rdone + t; r < rows; r += NTH) {  // unaligned rows (scalar)
+    double s = 0.0;
+    for (int q = 0; q < a.ninit; ++q) s += (double)__ldcs(in + q * a.init_stride + r);
+    out_row(r, s);
   }
   if (a.epi & 2) {
 #pragma unroll
