@@ -579,6 +579,17 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
   for (int q = 0; q < YASPMV_MAX_RANKS; ++q) a.peer_out[q] = nullptr;
   a.rcache = p.rc * p.C;
   a.tpc = A->tpc;
+  {  // warp-staged y stores (strategy 1, h = 1, no seg_row map, <= 40 KB of staging): on by
+     // default for the far part of a panel-sliced handle, whose slices hold ~1 block per row
+     // (C5: one scattered 4-byte store per row made a third of the far kernel's L2 requests;
+     // staged + streaming stores: 1.25 -> 1.13 ms); YASPMV_WSTAGE = 0 / 1 / 2 overrides
+    const char* e = std::getenv("YASPMV_WSTAGE");
+    const int want = e ? std::atoi(e) : (A->band_on ? 2 : 0);
+    a.wstage = (want && p.h == 1 && p.rc == 0 && !ablate && !(peers && p.S == 1) && c.n_zero == 0 &&
+                A->d.seg_row == nullptr && (int64_t)p.C * p.T * A->vsize <= 40 * 1024)
+                   ? want
+                   : 0;
+  }
   a.spin_limit = debug_spin_limit();
   a.spin_tile = debug_spin_slot();
   if (ablate && p.rc > 0) return fail(YASPMV_EUNSUPPORTED, "ablation / probe variants are strategy-1 kernels");

@@ -173,6 +173,10 @@ struct KArgs {
   // writes the waiting tile id to *spin_tile (mapped host memory) and traps
   long long spin_limit;
   long long* spin_tile;
+  // strategy 1, h = 1, no seg_row map: each warp stages its finished row sums in its slice of
+  // C*T values of dynamic shared memory and writes them as one contiguous run (the rows of a
+  // warp's stops are consecutive) instead of one scattered 4-byte store per row
+  int wstage;
 };
 
 // destinations of a fused exchange (combine kernel of BCCOO+, S > 1)

@@ -28,6 +28,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "common.hpp"
 #include "panel.hpp"
 
@@ -52,6 +54,11 @@ __device__ __forceinline__ uint32_t ld_flags16(const uint8_t* p) {
   return v;
 }
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ int ld_acquire_s32(const volatile int* p) {
+  int v;
+  asm volatile("ld.acquire.cta.shared::cta.b32 %0, [%1];" : "=r"(v) : "r"(smem_u32((const void*)p)) : "memory");
+  return v;
+}
 // acc slot of panel row r (identity: padded or permuted layouts that spread the warp's
 // stops, ~8 rows apart, over the banks cost more address arithmetic than the conflicts they
 // remove — measured 2.26 / 2.43 ms vs 2.15 ms on C5)
@@ -95,12 +102,13 @@ struct Layout {
   }
 };
 
-constexpr int NTH = PANEL_CTA, NWARP = NTH / 32, RING = 512, LAG = 128;
+constexpr int RING = 512, LAG = 128, MAXWARP = 32;
 static_assert(PANEL_TC == 512, "tile index = block offset >> 9");
-static_assert(RING > 2 * LAG + NWARP, "a look-back never reads a record slot that was reused");
+static_assert(RING > 2 * LAG + MAXWARP, "a look-back never reads a record slot that was reused");
 
 struct PanelShared {
   int sp[PANEL_MAX_KS + 2];        // slice_ptr of the panel (NS + 1 entries)
+  unsigned nemask[3];              // bit k: slice k is non-empty
   int fr[PANEL_MAX_KS + 1];        // first_row of every slice
   uint64_t bar[PANEL_NBUF];
   volatile int armed[PANEL_NBUF];  // window (non-empty band slice ordinal) armed on each buffer
@@ -111,7 +119,7 @@ struct PanelShared {
   float rT[RING];
   float rI[RING];
   volatile int rtag[RING];
-  double ss[NWARP];
+  double ss[MAXWARP];
 };
 
 // Thread 0 requests the x window of the o-th non-empty band slice of the panel (slices
@@ -148,8 +156,10 @@ __device__ __forceinline__ void issue_window(PanelShared& sh, unsigned char* buf
   sh.armed[o % PANEL_NBUF] = o;
 }
 
-template <typename VT>
+template <typename VT, int NTH>
 __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
+  constexpr int NWARP = NTH / 32;
+  static_assert(NWARP <= MAXWARP, "CTA size");
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ PanelShared sh;
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
@@ -174,6 +184,11 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     sh.sp[k] = a.slice_ptr[p * (KS + 1) + k];
     if (k < KS) sh.fr[k] = a.first_row[p * KS + k];
   }
+  if (t < 96) {  // bit k: slice k holds blocks (KS <= 64 band slices + the P7 far slice)
+    const bool ne = t < KS && a.slice_ptr[p * (KS + 1) + t] != a.slice_ptr[p * (KS + 1) + t + 1];
+    const unsigned b = __ballot_sync(0xffffffffu, ne);
+    if (lane == 0) sh.nemask[wid] = b;
+  }
   for (int q = t; q < RING; q += NTH) sh.rtag[q] = 0;
   if (t == 0) {
     for (int b = 0; b < PANEL_NBUF; ++b) {
@@ -187,9 +202,13 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   for (int r = t * (16 / (int)sizeof(VT)); r < R; r += NTH * (16 / (int)sizeof(VT)))
     *reinterpret_cast<uint4*>(acc + r) = make_uint4(0u, 0u, 0u, 0u);
   __syncthreads();
+  const unsigned long long nemask = ((unsigned long long)sh.nemask[1] << 32) | sh.nemask[0];
+  const unsigned nemask2 = sh.nemask[2];
   auto next_nonempty = [&](int k) {  // first slice >= k holding blocks (KS: none)
-    while (k < KS && sh.sp[k] == sh.sp[k + 1]) ++k;
-    return k;
+    const unsigned long long m = k < 64 ? nemask >> k : 0ull;
+    if (m) return k + __ffsll((long long)m) - 1;
+    const unsigned m2 = k < 96 ? nemask2 >> (max(k, 64) - 64) : 0u;
+    return m2 ? max(k, 64) + __ffs((int)m2) - 1 : KS;
   };
   auto issue = [&](int ow) { issue_window<VT>(sh, bufs, L.bufbytes, x, a.n, xe, cb, W, KS, fip, ow); };
   const int hf = fip && sh.sp[0] != sh.sp[1];  // the panel has a non-empty far slice (P7)
@@ -261,19 +280,29 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     // the low 16 bits and the has-stop flag above (a sum of flags is non-zero iff their OR is)
     int fn_ = nst | ((nst > 0) << 16);
     VT v = tail;
+    if (__ballot_sync(0xffffffffu, nst > 0) == 0xffffffffu) {
+      // every lane holds a stop (the common case): each lane's scanned value is its own
+      // tail, only the stop counts need the scan (the skip of P:222 at thread level)
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
-      const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
-      if (lane >= d) {
-        if (!(fn_ >> 16)) v = v2 + v;
-        fn_ += g2;
+      for (int d = 1; d < 32; d <<= 1) {
+        const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
+        if (lane >= d) fn_ += g2 & 0xFFFF;
+      }
+    } else {
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
+        const VT v2 = __shfl_up_sync(0xffffffffu, v, d);
+        if (lane >= d) {
+          if (!(fn_ >> 16)) v = v2 + v;
+          fn_ += g2;
+        }
       }
     }
     const int f = (fn_ >> 16) != 0;
-    prefetch();  // the warp's next tile in flight during this tile's updates and look-back
     // publish the tile's carry record (before anything waits on others); its carry-out is
-    // final at once when it holds a stop or starts its slice
+    // final at once when it holds a stop or starts its slice.  Before the next tile's loads
+    // are issued: the fence would otherwise wait for them to land
     const bool final_now = f || u == 0;
     if (lane == 31) {
       sh.rT[lt % RING] = v;  // inclusive: the tail after the tile's last stop, or its sum
@@ -281,6 +310,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       __threadfence_block();
       sh.rtag[lt % RING] = 2 * (lt + 1) + (final_now ? 1 : 0);
     }
+    prefetch();  // the warp's next tile in flight during this tile's updates and look-back
     const int gx = __shfl_up_sync(0xffffffffu, fn_, 1);
     int fx = (gx >> 16) != 0;
     int nx = gx & 0xFFFF;
@@ -338,10 +368,11 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
         int q = lt - 1;
         for (;; --q) {
           int tg;
-          while ((tg = sh.rtag[q % RING]) < 2 * (q + 1)) __nanosleep(16);
+          while ((tg = ld_acquire_s32(&sh.rtag[q % RING])) < 2 * (q + 1)) __nanosleep(16);
           if (tg & 1) break;
         }
-        __threadfence_block();
+        // acquire loads of the tags order the record reads (no fence: it would wait for
+        // the next tile's loads in flight)
         carry = sh.rI[q % RING];
         for (int r = q + 1; r < lt; ++r) carry = carry + sh.rT[r % RING];
       }
@@ -548,21 +579,44 @@ size_t panel_smem_bytes(int64_t R, int64_t W) {
   return (size_t)R * 4 + PANEL_NBUF * L.bufbytes;
 }
 
+// CTA size of the band kernel: PANEL_CTA, or YASPMV_PANEL_CTA in {512, 640, 704, 768, 896, 1024}
+// (exploration; registers per thread = 64K / size)
+static int panel_cta() {
+  static int c = [] {
+    const char* e = std::getenv("YASPMV_PANEL_CTA");
+    const int v = e ? std::atoi(e) : PANEL_CTA;
+    return (v == 512 || v == 640 || v == 704 || v == 768 || v == 896 || v == 1024) ? v : PANEL_CTA;
+  }();
+  return c;
+}
+template <typename F>
+static auto with_kernel(int nth, F&& f) {
+  switch (nth) {
+    case 512: return f(panel_kernel<float, 512>);
+    case 640: return f(panel_kernel<float, 640>);
+    case 704: return f(panel_kernel<float, 704>);
+    case 896: return f(panel_kernel<float, 896>);
+    case 1024: return f(panel_kernel<float, 1024>);
+    default: return f(panel_kernel<float, 768>);
+  }
+}
+
 int panel_attr(int64_t R, int64_t W, int* regs) {
-  cudaFuncAttributes fa;
-  cudaError_t e = cudaFuncGetAttributes(&fa, panel_kernel<float>);
-  if (e != cudaSuccess) return (int)e;
-  *regs = fa.numRegs;
-  int optin = 0, dev = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-  const size_t need = panel_smem_bytes(R, W);
-  if (need + fa.sharedSizeBytes > (size_t)optin) return (int)cudaErrorInvalidConfiguration;
-  e = cudaFuncSetAttribute(panel_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           optin - (int)fa.sharedSizeBytes);
-  if (e != cudaSuccess) return (int)e;
-  // two CTAs per SM when the windows allow it: the whole unified carve-out as shared memory
-  return (int)cudaFuncSetAttribute(panel_kernel<float>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  return with_kernel(panel_cta(), [&](auto kern) -> int {
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, kern);
+    if (e != cudaSuccess) return (int)e;
+    *regs = fa.numRegs;
+    int optin = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    const size_t need = panel_smem_bytes(R, W);
+    if (need + fa.sharedSizeBytes > (size_t)optin) return (int)cudaErrorInvalidConfiguration;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - (int)fa.sharedSizeBytes);
+    if (e != cudaSuccess) return (int)e;
+    // two CTAs per SM when the windows allow it: the whole unified carve-out as shared memory
+    return (int)cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  });
 }
 
 int launch_panel(const PanelArgs& a, int dtype, void* stream) {
@@ -571,9 +625,10 @@ int launch_panel(const PanelArgs& a, int dtype, void* stream) {
   // programmatic dependent launch (a.pdl): the CTAs may start while the far kernel's last
   // wave runs — that kernel lets dependents launch only after each of its CTAs has waited
   // for its own predecessors, so x is final; its results are read after this grid waits
+  const int nth = panel_cta();
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)a.npanels);
-  cfg.blockDim = dim3(NTH);
+  cfg.blockDim = dim3(nth);
   cfg.dynamicSmemBytes = panel_smem_bytes(a.R, a.W);
   cfg.stream = (cudaStream_t)stream;
   cudaLaunchAttribute attr[1];
@@ -581,7 +636,7 @@ int launch_panel(const PanelArgs& a, int dtype, void* stream) {
   attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return (int)cudaLaunchKernelEx(&cfg, panel_kernel<float>, a);
+  return with_kernel(nth, [&](auto kern) -> int { return (int)cudaLaunchKernelEx(&cfg, kern, a); });
 }
 
 }  // namespace yaspmv

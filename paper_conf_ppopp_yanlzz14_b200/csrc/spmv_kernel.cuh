@@ -512,6 +512,12 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   unsigned long long tk = 0;
   stream_tile<VT, H, W, T, CM, EPI>(a, tile, sh, t, C, fl, vw, xs, cta_seg0, tk);
   VT* out = static_cast<VT*>(a.out);
+  // warp-staged y stores (KArgs::wstage): this warp's slice of the dynamic shared memory
+  extern __shared__ __align__(16) unsigned char s1_stage[];
+  VT* const wbuf = (H == 1 && (EPI == 0 || EPI == 1) && a.wstage && a.seg_row == nullptr)
+                       ? reinterpret_cast<VT*>(s1_stage) + wid * 32 * T
+                       : nullptr;
+  const bool STG = wbuf != nullptr;
   // row stops: '0' bits; one popc gives their count
   const uint32_t stops = ~fl & TMASK;
   const int nst = __popc(stops);
@@ -664,6 +670,8 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
                 const VT o = (EPI == 1 || EPI == 2) ? run[r] * invv : run[r];
                 if (EPI == 3 && (a.ablate & ABL_NO_YSTORE)) {  // probe: the cost of the y stores
                   if (o == VT(-1.25e-30)) out[row * H + r] = o;
+                } else if (STG) {
+                  wbuf[nx + (int)(row - seg0)] = o;  // the warp's staging slice
                 } else {
                   store_out<VT, EPI>(a, out, row * H + r, o);
                 }
@@ -704,6 +712,18 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
         }
       }
     }
+  }
+  if (STG) {  // the warp's rows [cta_seg0 + Nw, + its stop count) as one contiguous run
+    __syncwarp();
+    const int wcnt = __shfl_sync(0xffffffffu, nn, 31);
+    const int skip = __ballot_sync(0xffffffffu, dependent) != 0u;  // slot 0: the carried segment
+    const int64_t wrow0 = (int64_t)cta_seg0 + Nw;
+    if (a.wstage == 2) {  // streaming stores (the slice results are read by a later kernel)
+      for (int i = lane + skip; i < wcnt; i += 32) __stcs(out + wrow0 + i, wbuf[i]);
+    } else {
+      for (int i = lane + skip; i < wcnt; i += 32) store_out<VT, EPI>(a, out, wrow0 + i, wbuf[i]);
+    }
+    __syncwarp();
   }
   double ss = (double)ssv;
 
@@ -986,13 +1006,22 @@ void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(C);
-  cfg.dynamicSmemBytes = TR::smem_bytes(C);
+  const size_t stage = a.wstage ? (size_t)C * T * H * sizeof(VT) : 0;
+  cfg.dynamicSmemBytes = TR::smem_bytes(C) + stage;
   cfg.stream = (cudaStream_t)stream;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  if (stage) {  // enough of the unified carve-out as shared memory for a full SM of CTAs (the
+                // instances prefer L1 otherwise, which would cap the CTAs per SM)
+    const size_t need = (size_t)(2048 / C) * (stage + 2048);
+    attr[1].id = cudaLaunchAttributePreferredSharedMemoryCarveout;
+    const size_t pct = (need * 100 + 228 * 1024 - 1) / (228 * 1024);
+    attr[1].val.sharedMemCarveout = (unsigned)(pct > 100 ? 100 : pct);
+    cfg.numAttrs = 2;
+  }
   // EPI: 0 plain SpMV, 1 power-iteration epilogue, 2 epilogue + peer stores (fused
   // exchange), 3 ablation / roofline probes (h = w = 1 only); separate instances so that
   // neither the peer loop nor the probes cost the production kernel registers
@@ -1020,7 +1049,12 @@ int attr_spmv(int C, int /*rc*/, int* regs, int* max_threads, int* blocks_per_sm
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     if (TR::smem_bytes(C) + fa.sharedSizeBytes > (size_t)optin) return 0;
-    e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TR::smem_bytes(C));
+    // the warp-staged y stores (KArgs::wstage) take up to 48 KB of dynamic shared memory on
+    // the EPI 0/1 instances: a fixed per-instance cap, whichever handle selects it
+    const int stage_cap = (int)(48 * 1024 - fa.sharedSizeBytes);
+    e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, max((int)TR::smem_bytes(C), stage_cap));
+    if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(k2, cudaFuncAttributeMaxDynamicSharedMemorySize, max((int)TR::smem_bytes(C), stage_cap));
     if (e != cudaSuccess) return (int)e;
     // x gathers are the L1 traffic: give L1 the whole unified carve-out
     e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
