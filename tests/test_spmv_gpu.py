@@ -317,3 +317,26 @@ def test_oracle_decode_matches_gpu_on_bccoo_plus():
         enc = E.encode(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, E.Params(1, 1, S, 8, 128, 0, 0))
         y, _ = _run(csr, x, S=S, T=8, C=128)
         assert np.array_equal(y.astype(np.float64), decode.spmv(enc, x))
+
+
+# ------------------------------------------------------------- warp-staged y stores (wstage)
+@pytest.mark.parametrize("params", [dict(T=8, C=256), dict(T=8, C=256, S=3), dict(T=16, C=128, tpc=2),
+                                    dict(T=4, C=64, S=2), dict(T=32, C=256)])
+def test_warp_staged_stores_bitwise(params, monkeypatch):
+    """KArgs::wstage (each warp's finished rows staged in shared memory and written as one
+    contiguous run, plain or streaming stores) writes exactly the values of the direct
+    per-row stores: y bitwise equal for wstage 0 / 1 / 2, and equal to the oracle's exact
+    integer result (integer-valued A, x), on a power-law matrix with empty rows, a long row
+    over many tiles (the carried segment's slot is skipped by the staged write-out) and
+    BCCOO+ slices."""
+    csr = synth.webbase_like(m=60000, integer=True)
+    x = np.random.default_rng(2).integers(-2, 3, csr.n).astype(np.float32)
+    exact = ref.spmv(csr.row_ptr, csr.col, csr.val, x)[0]
+    ys = []
+    for ws in ("0", "1", "2"):
+        monkeypatch.setenv("YASPMV_WSTAGE", ws)
+        y, _ = _run(csr, x, **params)
+        ys.append(y)
+    for y in ys[1:]:
+        assert np.array_equal(ys[0].view(np.uint32), y.view(np.uint32))
+    assert np.array_equal(ys[0].astype(np.float64), exact)
