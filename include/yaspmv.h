@@ -364,6 +364,28 @@ int64_t yaspmv_comm_seq(yaspmv_comm c);
 /* reports (and clears) a device-side wait timeout of an earlier step; synchronizes nothing. */
 yaspmv_status yaspmv_comm_check(yaspmv_comm c);
 int32_t yaspmv_launches_per_fused_step(yaspmv_matrix A);
+/* NVSwitch multicast for the fused step (not in the paper): instead of P
+ * stores of every finished row (one per rank's copy of x), ONE multimem.st through a
+ * multicast object to which every rank's x buffers are bound — the switch replicates it.
+ * Optional, after open_ipc / connect_local (the signal pads stay peer-mapped):
+ *   yaspmv_comm_mc_supported(device)  1 if the device reports switch multicast;
+ *   one rank: yaspmv_comm_mc_create(c, &fd)  multicast object for `world` devices, exported
+ *             as a POSIX file descriptor of the calling process (*fd_out);
+ *   the others: yaspmv_comm_mc_import(c, pid, fd)  the creator's pid and fd (duplicated with
+ *             pidfd_getfd, Linux >= 5.6; pid <= 0 or this process: dup(fd));
+ *   every rank: yaspmv_comm_mc_add_device(c); host barrier; yaspmv_comm_mc_bind(c) (allocates
+ *             2 x buffers of physical memory, binds them, maps them locally and through the
+ *             multicast object, copies the current x buffers in); host barrier.
+ * After bind, yaspmv_comm_x returns the bound buffers and every fused step stores through
+ * the multicast mapping.  Errors: YASPMV_EUNSUPPORTED without switch multicast or driver
+ * entry points, YASPMV_ECUDA with the CUresult of a failing driver call; a failed sequence
+ * leaves the comm on peer stores (mc_active = 0). */
+int32_t yaspmv_comm_mc_supported(int32_t device);
+yaspmv_status yaspmv_comm_mc_create(yaspmv_comm c, int64_t* fd_out);
+yaspmv_status yaspmv_comm_mc_import(yaspmv_comm c, int64_t pid, int64_t fd);
+yaspmv_status yaspmv_comm_mc_add_device(yaspmv_comm c);
+yaspmv_status yaspmv_comm_mc_bind(yaspmv_comm c);
+int32_t yaspmv_comm_mc_active(yaspmv_comm c);
 /* NULL-safe; unmaps the peers and frees the allocation (synchronize first; peers must not
  * write into this comm any more). */
 void yaspmv_comm_free(yaspmv_comm c);

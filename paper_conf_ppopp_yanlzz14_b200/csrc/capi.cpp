@@ -527,7 +527,9 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
     return YASPMV_OK;
   }
   if (c.ntiles == 0) {
-    if (peers)
+    if (peers && peers->mc)
+      launch_mc_zero(peers->p[0], c.m, A->vsize == 4 ? 0 : 1, cs);
+    else if (peers)
       for (int q = 0; q < peers->n; ++q) CUDA_TRY(cudaMemsetAsync(peers->p[q], 0, (size_t)c.m * A->vsize, cs));
     else
       CUDA_TRY(cudaMemsetAsync(y, 0, (size_t)c.m * A->vsize, cs));
@@ -576,6 +578,7 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
   a.pdl = (p.flags & YASPMV_NO_PDL) ? 0 : 1;
   a.dep_row = nullptr;
   a.npeer = 0;
+  a.peer_mc = 0;
   for (int q = 0; q < YASPMV_MAX_RANKS; ++q) a.peer_out[q] = nullptr;
   a.rcache = p.rc * p.C;
   a.tpc = A->tpc;
@@ -595,6 +598,7 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
   if (ablate && p.rc > 0) return fail(YASPMV_EUNSUPPORTED, "ablation / probe variants are strategy-1 kernels");
   if (peers && p.S == 1) {  // S > 1: the kernel writes tmp, the combine writes the peers
     a.npeer = peers->n;
+    a.peer_mc = peers->mc;
     for (int q = 0; q < peers->n; ++q) a.peer_out[q] = peers->p[q];
   }
   if (ablate & ABL_DEFER_CARRY) {
@@ -654,13 +658,16 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
     }
     return st;
   }
-  if (ablate || peers)
-    return fail(YASPMV_EUNSUPPORTED, "ablation variants and the fused exchange run the plain format only");
+  if (ablate) return fail(YASPMV_EUNSUPPORTED, "ablation variants run the plain format only");
+  if (peers && !A->pan.g.fip && !(A->can.p.S > 1 && A->can.ntiles > 0))
+    return fail(YASPMV_EUNSUPPORTED,
+                "fused exchange of a panel-sliced handle: the far part needs S > 1 (its slices stay in tmp) or P7");
   if (A->can.m == 0) {
     if (out_norm2) CUDA_TRY(cudaMemsetAsync(out_norm2, 0, sizeof(double), (cudaStream_t)stream));
     return YASPMV_OK;
   }
   DeviceGuard dg(A->device);
+  if (peers && peers->n > YASPMV_MAX_RANKS) return fail(YASPMV_EINVAL, "too many peers");
   if (ev) cudaEventRecord(ev[0], cs);
   // far part: BCCOO+ slices stay in tmp, the band kernel combines them (no combine kernel);
   // P7: the far entries are the panels' slice 0 — no far launch, acc starts at 0
@@ -703,6 +710,11 @@ yaspmv_status run_spmv(yaspmv_matrix A, const void* x, void* y, void* stream, co
   pa.pdl = (!fip && A->can.ntiles > 0 && !(A->can.p.flags & YASPMV_NO_PDL)) ? 1 : 0;
   pa.in_norm2 = in_norm2;
   pa.part = A->pd.part;
+  if (peers) {  // fused exchange: the band kernel's epilogue writes every rank's copy of x
+    pa.npeer = peers->n;
+    pa.peer_mc = peers->mc;
+    for (int q = 0; q < peers->n; ++q) pa.peer_out[q] = peers->p[q];
+  }
   const int e = launch_panel(pa, A->dtype, stream);
   if (e != 0) return fail(YASPMV_ECUDA, std::string("panel kernel: ") + cudaGetErrorString((cudaError_t)e));
   if (ev) cudaEventRecord(ev[2], cs);

@@ -13,7 +13,11 @@
 // peer stores into xbuf[(k+1)%2] of every rank -> ||z_k||^2 of the rank's rows -> publish
 // kernel: norm + flag = k+1 into every peer's pad, system-scope release after a
 // system-scope fence (the SpMV's peer stores precede it in stream order).
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <sys/syscall.h>
+#include <cerrno>
+#include <unistd.h>
 
 #include <algorithm>
 #include <cstring>
@@ -101,6 +105,65 @@ __global__ void wait_kernel(const char* __restrict__ sig, int world, unsigned lo
 }
 }  // namespace
 
+namespace {
+// CUDA driver entry points of the multicast path, resolved at run time through the runtime
+// (no link-time libcuda dependency)
+struct Drv {
+  bool ok = false;
+  CUresult (*devattr)(int*, CUdevice_attribute, CUdevice) = nullptr;
+  CUresult (*devget)(CUdevice*, int) = nullptr;
+  CUresult (*mc_gran)(size_t*, const CUmulticastObjectProp*, CUmulticastGranularity_flags) = nullptr;
+  CUresult (*mc_create)(CUmemGenericAllocationHandle*, const CUmulticastObjectProp*) = nullptr;
+  CUresult (*mc_add)(CUmemGenericAllocationHandle, CUdevice) = nullptr;
+  CUresult (*mc_bind)(CUmemGenericAllocationHandle, size_t, CUmemGenericAllocationHandle, size_t, size_t,
+                      unsigned long long) = nullptr;
+  CUresult (*mc_unbind)(CUmemGenericAllocationHandle, CUdevice, size_t, size_t) = nullptr;
+  CUresult (*mem_gran)(size_t*, const CUmemAllocationProp*, CUmemAllocationGranularity_flags) = nullptr;
+  CUresult (*mem_create)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*,
+                         unsigned long long) = nullptr;
+  CUresult (*mem_release)(CUmemGenericAllocationHandle) = nullptr;
+  CUresult (*addr_reserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long) = nullptr;
+  CUresult (*addr_free)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*mem_map)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long) = nullptr;
+  CUresult (*mem_unmap)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*set_access)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t) = nullptr;
+  CUresult (*export_h)(void*, CUmemGenericAllocationHandle, CUmemAllocationHandleType, unsigned long long) = nullptr;
+  CUresult (*import_h)(CUmemGenericAllocationHandle*, void*, CUmemAllocationHandleType) = nullptr;
+};
+template <typename F>
+bool entry(const char* name, F& f) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess ||
+      !p)
+    return false;
+  f = reinterpret_cast<F>(p);
+  return true;
+}
+const Drv& drv() {
+  static Drv d = [] {
+    Drv x;
+    x.ok = entry("cuDeviceGetAttribute", x.devattr) && entry("cuDeviceGet", x.devget) &&
+           entry("cuMulticastGetGranularity", x.mc_gran) && entry("cuMulticastCreate", x.mc_create) &&
+           entry("cuMulticastAddDevice", x.mc_add) && entry("cuMulticastBindMem", x.mc_bind) &&
+           entry("cuMulticastUnbind", x.mc_unbind) && entry("cuMemGetAllocationGranularity", x.mem_gran) &&
+           entry("cuMemCreate", x.mem_create) && entry("cuMemRelease", x.mem_release) &&
+           entry("cuMemAddressReserve", x.addr_reserve) && entry("cuMemAddressFree", x.addr_free) &&
+           entry("cuMemMap", x.mem_map) && entry("cuMemUnmap", x.mem_unmap) && entry("cuMemSetAccess", x.set_access) &&
+           entry("cuMemExportToShareableHandle", x.export_h) &&
+           entry("cuMemImportFromShareableHandle", x.import_h);
+    return x;
+  }();
+  return d;
+}
+}  // namespace
+
+#define CU_TRY(expr)                                                                         \
+  do {                                                                                       \
+    CUresult _r = (expr);                                                                    \
+    if (_r != CUDA_SUCCESS) return fail(YASPMV_ECUDA, std::string(#expr) + ": CUresult " + std::to_string((int)_r)); \
+  } while (0)
+
 struct yaspmv_comm_s {
   int device = -1, rank = 0, world = 1, dtype = 0, vsize = 4;
   int64_t chunk = 0, n_pad = 0;
@@ -117,11 +180,31 @@ struct yaspmv_comm_s {
   int* d_err = nullptr;
   int64_t scratch_n = 0;
   double* d_scratch = nullptr;
+  // NVSwitch multicast (yaspmv_comm_mc_*): the two x buffers live in a VMM allocation bound
+  // to a multicast object of all ranks; the SpMV stores z through the multicast mapping
+  bool mc = false;                         // bound: steps use mc_va / loc_va
+  bool mc_have = false, mc_added = false, mem_have = false;
+  CUmemGenericAllocationHandle mc_h = 0, mem_h = 0;
+  size_t mc_size = 0;
+  CUdeviceptr mc_va = 0, loc_va = 0;
+  int mc_fd = -1;
   ~yaspmv_comm_s() {
     if (device < 0) return;
     int cur = 0;
     cudaGetDevice(&cur);
     cudaSetDevice(device);
+    if (mc_have || mem_have) {
+      cudaDeviceSynchronize();
+      const Drv& d = drv();
+      CUdevice dev = 0;
+      d.devget(&dev, device);
+      if (mc_va) { d.mem_unmap(mc_va, mc_size); d.addr_free(mc_va, mc_size); }
+      if (loc_va) { d.mem_unmap(loc_va, mc_size); d.addr_free(loc_va, mc_size); }
+      if (mc && mc_have) d.mc_unbind(mc_h, dev, 0, mc_size);
+      if (mem_have) d.mem_release(mem_h);
+      if (mc_have) d.mem_release(mc_h);
+    }
+    if (mc_fd >= 0) close(mc_fd);
     for (int q = 0; q < MAXR; ++q)
       if (ipc[q] && peer[q]) cudaIpcCloseMemHandle(peer[q]);
     if (base) cudaFree(base);
@@ -131,6 +214,7 @@ struct yaspmv_comm_s {
     cudaSetDevice(cur);
   }
   char* xbuf(const char* b, int64_t k) const { return const_cast<char*>(b) + (size_t)(k & 1) * xbytes; }
+  char* xown() const { return mc ? reinterpret_cast<char*>(loc_va) : base; }  // this rank's x buffers
   char* sig(const char* b) const { return const_cast<char*>(b) + 2 * xbytes; }
 };
 
@@ -232,8 +316,131 @@ yaspmv_status yaspmv_comm_connect_local(yaspmv_comm c, const yaspmv_comm* peers,
 
 void* yaspmv_comm_x(yaspmv_comm c, int32_t which) {
   if (!c) return nullptr;
-  return c->xbuf(c->base, c->seq + (which & 1));
+  return c->xbuf(c->xown(), c->seq + (which & 1));
 }
+
+// ---- NVSwitch multicast: one multimem.st per element instead of P stores
+int32_t yaspmv_comm_mc_supported(int32_t device) {
+  const Drv& d = drv();
+  if (!d.ok) return 0;
+  CUdevice dev = 0;
+  int v = 0;
+  if (d.devget(&dev, device) != CUDA_SUCCESS) return 0;
+  if (d.devattr(&v, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, dev) != CUDA_SUCCESS) return 0;
+  return v ? 1 : 0;
+}
+
+static size_t mc_bytes(yaspmv_comm c, size_t* gran_out) {
+  const Drv& d = drv();
+  CUmulticastObjectProp mp = {};
+  mp.numDevices = (unsigned)c->world;
+  mp.size = 2 * c->xbytes;
+  mp.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+  size_t g1 = 0, g2 = 0;
+  d.mc_gran(&g1, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED);
+  CUmemAllocationProp ap = {};
+  ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ap.location.id = c->device;
+  d.mem_gran(&g2, &ap, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED);
+  size_t g = std::max<size_t>(std::max(g1, g2), 2u << 20);
+  *gran_out = g;
+  return round_up(2 * c->xbytes, g);
+}
+
+yaspmv_status yaspmv_comm_mc_create(yaspmv_comm c, int64_t* fd_out) {
+  if (!c || !fd_out) return fail(YASPMV_EINVAL, "NULL argument");
+  if (!yaspmv_comm_mc_supported(c->device)) return fail(YASPMV_EUNSUPPORTED, "device has no switch multicast");
+  if (c->mc_have) return fail(YASPMV_EINVAL, "multicast object already present");
+  const Drv& d = drv();
+  CUDA_TRY(cudaSetDevice(c->device));
+  size_t g = 0;
+  c->mc_size = mc_bytes(c, &g);
+  CUmulticastObjectProp mp = {};
+  mp.numDevices = (unsigned)c->world;
+  mp.size = c->mc_size;
+  mp.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+  CU_TRY(d.mc_create(&c->mc_h, &mp));
+  c->mc_have = true;
+  int fd = -1;
+  CU_TRY(d.export_h(&fd, c->mc_h, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0));
+  c->mc_fd = fd;
+  *fd_out = fd;
+  return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_comm_mc_import(yaspmv_comm c, int64_t pid, int64_t fd) {
+  if (!c) return fail(YASPMV_EINVAL, "NULL comm");
+  if (c->mc_have) return fail(YASPMV_EINVAL, "multicast object already present");
+  const Drv& d = drv();
+  if (!d.ok) return fail(YASPMV_EUNSUPPORTED, "driver multicast entry points unavailable");
+  CUDA_TRY(cudaSetDevice(c->device));
+  size_t g = 0;
+  c->mc_size = mc_bytes(c, &g);
+  int local = -1;
+  if (pid <= 0 || pid == (int64_t)getpid()) {
+    local = dup((int)fd);
+  } else {  // the creator's descriptor, duplicated into this process (Linux >= 5.6)
+    const int pfd = (int)syscall(SYS_pidfd_open, (pid_t)pid, 0);
+    if (pfd < 0) return fail(YASPMV_ECUDA, "pidfd_open failed (errno " + std::to_string(errno) + ")");
+    local = (int)syscall(SYS_pidfd_getfd, pfd, (int)fd, 0);
+    close(pfd);
+  }
+  if (local < 0) return fail(YASPMV_ECUDA, "could not obtain the multicast descriptor (errno " + std::to_string(errno) + ")");
+  c->mc_fd = local;
+  CU_TRY(d.import_h(&c->mc_h, (void*)(uintptr_t)local, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR));
+  c->mc_have = true;
+  return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_comm_mc_add_device(yaspmv_comm c) {
+  if (!c || !c->mc_have) return fail(YASPMV_EINVAL, "no multicast object (mc_create / mc_import first)");
+  if (c->mc_added) return YASPMV_OK;
+  const Drv& d = drv();
+  CUDA_TRY(cudaSetDevice(c->device));
+  CUdevice dev = 0;
+  CU_TRY(d.devget(&dev, c->device));
+  CU_TRY(d.mc_add(c->mc_h, dev));
+  c->mc_added = true;
+  return YASPMV_OK;
+}
+
+yaspmv_status yaspmv_comm_mc_bind(yaspmv_comm c) {
+  if (!c || !c->mc_added) return fail(YASPMV_EINVAL, "mc_add_device first (on every rank)");
+  if (c->mc) return YASPMV_OK;
+  const Drv& d = drv();
+  CUDA_TRY(cudaSetDevice(c->device));
+  CUdevice dev = 0;
+  CU_TRY(d.devget(&dev, c->device));
+  size_t g = 0;
+  const size_t sz = mc_bytes(c, &g);
+  if (sz != c->mc_size) return fail(YASPMV_EINVAL, "multicast size mismatch between ranks");
+  CUmemAllocationProp ap = {};
+  ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ap.location.id = c->device;
+  CU_TRY(d.mem_create(&c->mem_h, sz, &ap, 0));
+  c->mem_have = true;
+  CU_TRY(d.mc_bind(c->mc_h, 0, c->mem_h, 0, sz, 0));
+  CUmemAccessDesc acc = {};
+  acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  acc.location.id = c->device;
+  acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  CU_TRY(d.addr_reserve(&c->loc_va, sz, g, 0, 0));
+  CU_TRY(d.mem_map(c->loc_va, sz, 0, c->mem_h, 0));
+  CU_TRY(d.set_access(c->loc_va, sz, &acc, 1));
+  CU_TRY(d.addr_reserve(&c->mc_va, sz, g, 0, 0));
+  CU_TRY(d.mem_map(c->mc_va, sz, 0, c->mc_h, 0));
+  CU_TRY(d.set_access(c->mc_va, sz, &acc, 1));
+  // the current x buffers move into the bound memory; from here on steps read loc_va and
+  // store through mc_va
+  CUDA_TRY(cudaMemcpy(reinterpret_cast<void*>(c->loc_va), c->base, 2 * c->xbytes, cudaMemcpyDeviceToDevice));
+  CUDA_TRY(cudaDeviceSynchronize());
+  c->mc = true;
+  return YASPMV_OK;
+}
+
+int32_t yaspmv_comm_mc_active(yaspmv_comm c) { return c && c->mc ? 1 : 0; }
 
 yaspmv_status yaspmv_comm_begin(yaspmv_comm c) {
   if (!c) return fail(YASPMV_EINVAL, "NULL comm");
@@ -282,10 +489,16 @@ yaspmv_status yaspmv_power_step_fused(yaspmv_matrix A, yaspmv_comm c, void* stre
     if (st != YASPMV_OK) return st;
   }
   PeerOut po;
-  po.n = c->world;
-  for (int q = 0; q < c->world; ++q)
-    po.p[q] = c->xbuf(c->peer[q], c->seq + 1) + (size_t)c->rank * c->chunk * c->vsize;
-  yaspmv_status st = run_spmv_peers(A, c->xbuf(c->base, c->seq), scaled ? c->d_norm_local + 1 : nullptr,
+  if (c->mc) {  // one multimem.st per element: the switch writes every rank's buffer
+    po.n = 1;
+    po.mc = 1;
+    po.p[0] = c->xbuf(reinterpret_cast<const char*>(c->mc_va), c->seq + 1) + (size_t)c->rank * c->chunk * c->vsize;
+  } else {
+    po.n = c->world;
+    for (int q = 0; q < c->world; ++q)
+      po.p[q] = c->xbuf(c->peer[q], c->seq + 1) + (size_t)c->rank * c->chunk * c->vsize;
+  }
+  yaspmv_status st = run_spmv_peers(A, c->xbuf(c->xown(), c->seq), scaled ? c->d_norm_local + 1 : nullptr,
                                     c->d_norm_local, po, stream);
   if (st != YASPMV_OK) return st;
   PeerSig ps;

@@ -167,6 +167,7 @@ struct KArgs {
   // pre-offset to this rank's chunk) instead of out[i]
   int npeer;
   void* peer_out[YASPMV_MAX_RANKS];
+  int peer_mc;             // 1: peer_out[0] is a multicast address (npeer = 1, multimem.st)
   int rcache;              // strategy 2: result cache entries (rc * C); 0 for strategy 1
   int tpc;                 // consecutive tiles per workgroup (block-id mode); grid = ceil(ntiles / tpc)
   // debug spin bound: > 0 = a look-back that polls more than spin_limit times
@@ -179,11 +180,25 @@ struct KArgs {
   int wstage;
 };
 
-// destinations of a fused exchange (combine kernel of BCCOO+, S > 1)
+// destinations of a fused exchange (combine kernel of BCCOO+, S > 1); mc = 1: p[0] is an
+// NVSwitch multicast address (n = 1) — one multimem.st reaches every rank's buffer
 struct PeerOut {
   int n = 0;
+  int mc = 0;
   void* p[YASPMV_MAX_RANKS] = {};
 };
+
+#ifdef __CUDACC__
+// one store through a multicast mapping (multimem.st, sm_90+): the switch writes it into
+// every bound buffer
+template <typename VT>
+__device__ __forceinline__ void multimem_store(VT* p, VT v) {
+  if constexpr (sizeof(VT) == 4)
+    asm volatile("multimem.st.relaxed.sys.global.f32 [%0], %1;" ::"l"(p), "f"((float)v) : "memory");
+  else
+    asm volatile("multimem.st.relaxed.sys.global.f64 [%0], %1;" ::"l"(p), "d"((double)v) : "memory");
+}
+#endif
 
 typedef void (*LaunchFn)(const KArgs& a, int C, int64_t grid, void* stream);
 typedef int (*AttrFn)(int C, int rc, int* regs, int* max_threads, int* blocks_per_sm);
@@ -198,6 +213,7 @@ struct KernelEntry {
 const KernelEntry* find_kernel(int dtype, int h, int w, int T, int cm, int strat = 1);
 const std::vector<KernelEntry>& all_kernels();
 
+void launch_mc_zero(void* p, int64_t n, int dtype, void* stream);
 void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, int dtype, void* stream,
                     const double* in_norm2 = nullptr, double* part = nullptr, const PeerOut* peers = nullptr);
 int64_t combine_blocks(int64_t m);

@@ -2,6 +2,7 @@
 // registry of precompiled SpMV instances.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <mutex>
 
 #include "common.hpp"
@@ -25,7 +26,9 @@ __global__ void combine_kernel(const VT* __restrict__ tmp, VT* __restrict__ y, i
     double s = (double)__ldcs(tmp + i);
     for (int q = 1; q < S; ++q) s += (double)__ldcs(tmp + (int64_t)q * stride + i);
     const VT o = in_norm2 ? (VT)((VT)s * inv) : (VT)s;
-    if (peers.n > 0) {  // fused exchange: every rank's copy of the next x (yaspmv_power_step_fused)
+    if (peers.mc) {  // fused exchange through an NVSwitch multicast mapping
+      multimem_store(static_cast<VT*>(peers.p[0]) + i, o);
+    } else if (peers.n > 0) {  // fused exchange: every rank's copy of the next x (yaspmv_power_step_fused)
 #pragma unroll
       for (int q = 0; q < YASPMV_MAX_RANKS; ++q)
         if (q < peers.n) static_cast<VT*>(peers.p[q])[i] = o;
@@ -69,6 +72,20 @@ void launch_combine(const void* tmp, void* y, int64_t m, int64_t stride, int S, 
   else
     combine_kernel<double><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>((const double*)tmp, (double*)y, m,
                                                                                stride, S, in_norm2, part, po);
+}
+
+// zeros through a multicast mapping (an empty matrix in a fused step: cudaMemset does not take
+// multicast addresses)
+template <typename VT>
+__global__ void mc_zero_kernel(VT* p, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    multimem_store(p + i, VT(0));
+}
+void launch_mc_zero(void* p, int64_t n, int dtype, void* stream) {
+  if (n <= 0) return;
+  const unsigned blocks = (unsigned)std::min<int64_t>((n + 255) / 256, 1184);
+  if (dtype == 0) mc_zero_kernel<float><<<blocks, 256, 0, (cudaStream_t)stream>>>((float*)p, n);
+  else mc_zero_kernel<double><<<blocks, 256, 0, (cudaStream_t)stream>>>((double*)p, n);
 }
 
 // ---------------------------------------------------------------- ||v||^2

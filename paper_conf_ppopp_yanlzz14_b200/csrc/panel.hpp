@@ -113,6 +113,12 @@ struct PanelArgs {
   int pdl;            // launched as a programmatic dependent of the far kernel (see launch_panel)
   const double* in_norm2;
   double* part;
+  // fused exchange (yaspmv_power_step_fused): npeer > 0 writes y to peer_out[q] for q < npeer
+  // (every rank's copy of the next x) instead of y; peer_mc: peer_out[0] is a multicast
+  // address (one multimem.st per element)
+  int npeer = 0;
+  int peer_mc = 0;
+  void* peer_out[YASPMV_MAX_RANKS] = {};
 };
 // panel_kernel.cu
 int launch_panel(const PanelArgs& a, int dtype, void* stream);  // returns cudaError_t

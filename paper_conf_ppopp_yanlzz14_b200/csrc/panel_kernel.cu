@@ -493,16 +493,39 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   if (a.pdl && a.ninit > 0) cudaGridDependencySynchronize();  // the far kernel is complete
   const double inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
   const VT* in = static_cast<const VT*>(a.init) + row0;
+  // the output: y, or in a fused exchange every rank's copy of the next x (peer stores, or one
+  // store through a multicast mapping)
+  auto store_y = [&](int64_t i, VT v) {
+    if (a.peer_mc) {
+      multimem_store(static_cast<VT*>(a.peer_out[0]) + i, v);
+    } else if (a.npeer > 0) {
+      for (int q = 0; q < a.npeer; ++q) static_cast<VT*>(a.peer_out[q])[i] = v;
+    } else {
+      y[i] = v;
+    }
+  };
+  auto store_y4 = [&](int64_t i, float4 v) {
+    if (a.peer_mc) {
+      asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(static_cast<float*>(a.peer_out[0]) + i),
+                   "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+                   : "memory");
+    } else if (a.npeer > 0) {
+      for (int q = 0; q < a.npeer; ++q) *reinterpret_cast<float4*>(static_cast<float*>(a.peer_out[q]) + i) = v;
+    } else {
+      *reinterpret_cast<float4*>(y + i) = v;
+    }
+  };
   // y[r] = (VT)((s_0 + ... + s_{S-1} in fp64, ascending) + acc[r]) * inv)
   auto out_row = [&](int r, double s) {
     const VT o2 = a.ninit > 0 ? (VT)((s + (double)acc[swz(r)]) * inv)
                               : ((a.epi & 1) ? (VT)(acc[swz(r)] * inv) : acc[swz(r)]);
-    y[row0 + r] = o2;
+    store_y(row0 + r, o2);
     ssq += (double)o2 * (double)o2;
   };
   int rdone = 0;
-  if (sizeof(VT) == 4 && ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(y + row0)) & 15) == 0 &&
-      (a.init_stride & 3) == 0) {
+  uintptr_t oal = a.npeer > 0 ? 0 : reinterpret_cast<uintptr_t>(y + row0);
+  for (int q = 0; q < a.npeer; ++q) oal |= reinterpret_cast<uintptr_t>(static_cast<VT*>(a.peer_out[q]) + row0);
+  if (sizeof(VT) == 4 && ((reinterpret_cast<uintptr_t>(in) | oal) & 15) == 0 && (a.init_stride & 3) == 0) {
     // 128-bit loads of the far part's slice results, every slice of two row quads in flight
     // at once (the epilogue runs with no other CTA on the SM to hide its latency)
     const int ng = rows >> 2;
@@ -548,7 +571,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
             ssq += (double)oi[j] * (double)oi[j];
           }
           o = make_float4(oi[0], oi[1], oi[2], oi[3]);
-          *reinterpret_cast<float4*>(y + row0 + 4 * g) = o;
+          store_y4(row0 + 4 * g, o);
         }
       }
     }

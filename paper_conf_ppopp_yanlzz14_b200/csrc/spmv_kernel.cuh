@@ -201,6 +201,10 @@ __device__ __forceinline__ double ld_relaxed_f64(const double* p) {
 template <typename VT, int EPI>
 __device__ __forceinline__ void store_out(const KArgs& a, VT* out, int64_t i, VT v) {
   if constexpr (EPI == 2) {
+    if (a.peer_mc) {  // NVSwitch multicast: one store, every rank's copy
+      multimem_store(static_cast<VT*>(a.peer_out[0]) + i, v);
+      return;
+    }
 #pragma unroll
     for (int q = 0; q < YASPMV_MAX_RANKS; ++q)
       if (q < a.npeer) static_cast<VT*>(a.peer_out[q])[i] = v;

@@ -183,13 +183,14 @@ class FusedPowerIteration:
     class (CPU tests of the exchange logic)."""
 
     def __init__(self, layout: Layout, A, dtype, device, group=None, comm=None, timeout_ms: int = 0,
-                 comm_factory=None):
+                 comm_factory=None, multicast=False):
         import torch
         self.L = layout
         self.A = A
         self.group = group
         self.device = torch.device(device)
         self.own_comm = comm is None
+        self.multicast = False
         if comm is None:
             if comm_factory is None:
                 from .matrix import Comm as comm_factory
@@ -228,8 +229,51 @@ class FusedPowerIteration:
                     raise
             elif err is not None:
                 raise err
+            if multicast:
+                self._setup_multicast(comm, layout, group, required=multicast is True)
         self.comm = comm
         self.restart()
+
+    def _setup_multicast(self, comm, layout, group, required):
+        """NVSwitch multicast (yaspmv_comm_mc_*): rank 0 creates the multicast object and
+        exports it as a POSIX fd, the others duplicate it (pidfd_getfd), every rank adds its
+        device, then every rank binds its x buffers; from then on each step stores z once
+        through the multicast mapping instead of once per rank.  Every stage is agreed on;
+        ``required`` False (multicast="auto") keeps the peer stores if any rank fails."""
+        import os
+        world = layout.world
+        def stage(fn, what):
+            err = None
+            try:
+                out = fn()
+            except Exception as e:
+                out, err = None, e
+            if world > 1:
+                self._agree(err, group, what)
+            elif err is not None:
+                raise RuntimeError(f"fused exchange: could not {what}: {err}")
+            return out
+        def probe():
+            if not comm.mc_supported(self.device.index or 0):
+                raise RuntimeError("the device reports no switch multicast")
+        try:
+            stage(probe, "use switch multicast")
+            mine = stage(lambda: (os.getpid(), comm.mc_create()) if layout.rank == 0 else None,
+                         "create the multicast object")
+            if world > 1:
+                import torch.distributed as dist
+                infos = [None] * world
+                dist.all_gather_object(infos, mine, group=group)
+                pid, fd = infos[0]
+            else:
+                pid, fd = mine
+            stage(lambda: None if layout.rank == 0 else comm.mc_import(pid, fd), "import the multicast object")
+            stage(comm.mc_add_device, "add the devices to the multicast object")
+            stage(comm.mc_bind, "bind the x buffers to the multicast object")
+        except RuntimeError:
+            if required:
+                raise
+        self.multicast = bool(getattr(comm, "mc_active", False))
 
     @staticmethod
     def _agree(err, group, what):

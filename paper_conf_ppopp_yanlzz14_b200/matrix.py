@@ -230,6 +230,30 @@ class Comm:
         arr = (ctypes.c_void_p * len(peers))(*[p._h.value for p in peers])
         check(lib.yaspmv_comm_connect_local(self._h, arr, len(peers)))
 
+    # ---- NVSwitch multicast (include/yaspmv.h "yaspmv_comm_mc_*")
+    @staticmethod
+    def mc_supported(device: int) -> bool:
+        return bool(lib.yaspmv_comm_mc_supported(device))
+
+    def mc_create(self) -> int:
+        """Creator rank: the multicast object for `world` devices; returns its POSIX fd."""
+        fd = ctypes.c_int64()
+        check(lib.yaspmv_comm_mc_create(self._h, ctypes.byref(fd)))
+        return fd.value
+
+    def mc_import(self, pid: int, fd: int) -> None:
+        check(lib.yaspmv_comm_mc_import(self._h, pid, fd))
+
+    def mc_add_device(self) -> None:
+        check(lib.yaspmv_comm_mc_add_device(self._h))
+
+    def mc_bind(self) -> None:
+        check(lib.yaspmv_comm_mc_bind(self._h))
+
+    @property
+    def mc_active(self) -> bool:
+        return bool(lib.yaspmv_comm_mc_active(self._h))
+
     def x(self, which: int = 0):
         """torch view of x buffer (seq + which) % 2 (which = 0: the next step's input /
         the latest z; 1: the buffer the next step writes), world * chunk elements."""

@@ -93,15 +93,19 @@ def _fused_local(Ls, As, tdt, iters):
     return out, comms
 
 
+BAND = dict(B=4096, R=4096, W=4096, S=2, T=16, C=128)  # panel-sliced BCCOO+ (DESIGN §2.1), far part S = 2
+
+
 @pytest.mark.parametrize("P", [1, 2, 3])
-@pytest.mark.parametrize("case", ["circuit-f32", "circuit-f32-S2", "laplace-f64"])
+@pytest.mark.parametrize("case", ["circuit-f32", "circuit-f32-S2", "laplace-f64", "circuit-band"])
 def test_fused_step_bitwise_equals_unfused(P, case):
     _need_gpu()
     from synth import matrices as sm
     if case.startswith("circuit"):
         csr = sm.circuit_like_rows(0, KW["n"], **KW)
         tdt = torch.float32
-        params = dict(T=16, C=128, S=2) if case.endswith("S2") else dict(T=16, C=128)
+        params = (dict(T=16, C=128, S=2) if case.endswith("S2") else BAND if case.endswith("band")
+                  else dict(T=16, C=128))
     else:
         csr = synth.laplacian_2d(64)
         tdt = torch.float64
@@ -206,7 +210,7 @@ def _free_port():
     return p
 
 
-def _ipc_worker(rank, world, port, path, iters, per_rank_device=False):
+def _ipc_worker(rank, world, port, path, iters, per_rank_device=False, multicast=False):
     import torch.distributed as dist
     from synth import matrices as sm
     from paper_conf_ppopp_yanlzz14_b200 import Matrix, dist as D
@@ -220,7 +224,9 @@ def _ipc_worker(rank, world, port, path, iters, per_rank_device=False):
     sub = csr.row_slice(L.r0, L.r1)
     A = Matrix.from_csr(sub.m, L.n_padded, sub.row_ptr, D.remap_columns(sub.col, L.bounds, L.m_max), sub.val,
                         device=dev, T=16, C=128)
-    pit = D.FusedPowerIteration(L, A, torch.float32, f"cuda:{dev}", timeout_ms=60000)  # IPC handle exchange
+    pit = D.FusedPowerIteration(L, A, torch.float32, f"cuda:{dev}", timeout_ms=60000,  # IPC handle exchange
+                                multicast=multicast)
+    assert pit.multicast == bool(multicast)
     for _ in range(iters):
         pit.step()
     pit.comm.wait()
@@ -249,6 +255,77 @@ def test_fused_two_processes_ipc(two_devices):
     with tempfile.TemporaryDirectory() as td:
         path = os.path.join(td, "z")
         mp.spawn(_ipc_worker, args=(2, _free_port(), path, iters, two_devices), nprocs=2, join=True)
+        zs = [np.load(path + f".{r}.npy") for r in range(2)]
+        n2 = [np.load(path + f".{r}.n2.npy") for r in range(2)]
+    csr = sm.circuit_like_rows(0, KW["n"], **KW)
+    Ls, As = _rank_matrices(csr, 2, dict(T=16, C=128))
+    x_ref, tot_ref = _unfused_reference(Ls, As, torch.float32, iters)
+    for r in range(2):
+        assert np.array_equal(zs[r], x_ref.cpu().numpy())
+        assert np.array_equal(n2[r], tot_ref.cpu().numpy())
+
+
+def _mc_supported():
+    from paper_conf_ppopp_yanlzz14_b200 import Comm
+    return Comm.mc_supported(0)
+
+
+@pytest.mark.parametrize("case", ["circuit-f32", "circuit-f32-S2", "laplace-f64", "circuit-band"])
+def test_fused_multicast_one_rank(case):
+    """NVSwitch multicast exchange (yaspmv_comm_mc_*): the multicast object of one device,
+    the x buffers bound to it, every z row stored once through the multicast mapping by the
+    SpMV epilogue (S = 1) or the BCCOO+ combine (S = 2) — bitwise equal to the unfused
+    protocol.  The object, the binding and the multimem.st path are the ones a multi-GPU
+    node uses (there the switch replicates each store into every rank's buffer)."""
+    _need_gpu()
+    if not _mc_supported():
+        pytest.skip("the device reports no switch multicast")
+    from synth import matrices as sm
+    from paper_conf_ppopp_yanlzz14_b200 import dist as D
+    if case.startswith("circuit"):
+        csr = sm.circuit_like_rows(0, KW["n"], **KW)
+        tdt = torch.float32
+        params = (dict(T=16, C=128, S=2) if case.endswith("S2") else BAND if case.endswith("band")
+                  else dict(T=16, C=128))
+    else:
+        csr = synth.laplacian_2d(64)
+        tdt = torch.float64
+        params = dict(T=8, C=64)
+    iters = 4
+    Ls, As = _rank_matrices(csr, 1, params)
+    x_ref, tot_ref = _unfused_reference(Ls, As, tdt, iters)
+    try:
+        pit = D.FusedPowerIteration(Ls[0], As[0], tdt, "cuda:0", timeout_ms=20000, multicast=True)
+    except RuntimeError as e:  # e.g. a container without the switch's fabric channels
+        if "create the multicast object" in str(e):
+            pytest.skip(f"the driver refuses multicast objects here: {e}")
+        raise
+    assert pit.multicast and pit.comm.mc_active
+    for _ in range(iters):
+        pit.step()
+    pit.comm.wait()
+    torch.cuda.synchronize()
+    pit.comm.check()
+    assert torch.equal(pit.comm.x(0), x_ref)
+    assert torch.equal(pit.comm.norm2(), tot_ref)
+    pit.comm.free()
+    for A in As:
+        A.free()
+
+
+def test_fused_two_processes_multicast():
+    """Two processes on two GPUs, the multicast object created by rank 0 and imported by
+    rank 1 through pidfd_getfd: every z row crosses the switch once.  Runs only where two
+    GPUs with switch multicast are visible."""
+    _need_gpu()
+    if torch.cuda.device_count() < 2 or not _mc_supported():
+        pytest.skip("needs two visible GPUs with switch multicast")
+    import torch.multiprocessing as mp
+    from synth import matrices as sm
+    iters = 3
+    with tempfile.TemporaryDirectory() as td:
+        path = os.path.join(td, "z")
+        mp.spawn(_ipc_worker, args=(2, _free_port(), path, iters, True, True), nprocs=2, join=True)
         zs = [np.load(path + f".{r}.npy") for r in range(2)]
         n2 = [np.load(path + f".{r}.n2.npy") for r in range(2)]
     csr = sm.circuit_like_rows(0, KW["n"], **KW)
