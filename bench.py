@@ -31,7 +31,9 @@ sys.path.insert(0, ROOT)
 
 # tuned defaults per config (yaspmv_tune on B200)
 DEFAULT_PARAMS = {
-    "c5": dict(h=1, w=1, S=3, T=8, C=256, col_mode=2, B=65536, R=16384, W=16384),
+    # C5: band kernel on panels of 16128 rows (3,101 panels = 20.95 waves of 148 SMs; 9 slices of
+    # 16384 columns); far part BCCOO+ S = 3, T = 8, C = 128, 4 tiles per CTA (profiles/r05_*)
+    "c5": dict(h=1, w=1, S=3, T=8, C=128, tpc=4, col_mode=2, B=65536, R=16128, W=16384),
     "c4": dict(h=1, w=1, S=1, T=16, C=256),
     "c3-spheres": dict(h=4, w=4, T=4, C=128),
     "c3-cantilever": dict(h=4, w=4, T=4, C=128),

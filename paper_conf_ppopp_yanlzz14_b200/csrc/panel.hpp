@@ -24,8 +24,9 @@ namespace yaspmv {
 constexpr int PANEL_BT = 16;
 constexpr int PANEL_WT = 32;
 constexpr int PANEL_TC = PANEL_BT * PANEL_WT;
-constexpr int PANEL_CTA = 768;       // 24 warps, <= 80 registers (measured: 512 / 768 / 896 / 1024
-                                      // threads -> 2.21 / 2.07 / 2.13 / 2.16 ms on C5)
+constexpr int PANEL_CTA = 640;       // 20 warps, <= 96 registers; C5 band kernel after the round-2
+                                      // changes, 640 / 704 / 768 / 896 / 1024 threads -> 1.875 (R =
+                                      // 16128) / 1.99 / 1.91 / 1.94 / 2.28 ms (YASPMV_PANEL_CTA)
 constexpr int PANEL_MAX_KS = 64;      // slices per panel
 constexpr int PANEL_NBUF = 2;         // x windows resident per CTA (current + next slice)
 
