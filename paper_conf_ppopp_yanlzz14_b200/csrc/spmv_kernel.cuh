@@ -1018,13 +1018,26 @@ void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
   attr[0].val.programmaticStreamSerializationAllowed = a.pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (stage) {  // enough of the unified carve-out as shared memory for a full SM of CTAs (the
-                // instances prefer L1 otherwise, which would cap the CTAs per SM)
-    const size_t need = (size_t)(2048 / C) * (stage + 2048);
-    attr[1].id = cudaLaunchAttributePreferredSharedMemoryCarveout;
-    const size_t pct = (need * 100 + 228 * 1024 - 1) / (228 * 1024);
-    attr[1].val.sharedMemCarveout = (unsigned)(pct > 100 ? 100 : pct);
-    cfg.numAttrs = 2;
+  {  // staged stores need enough of the unified carve-out as shared memory for a full SM of
+     // CTAs (the instances prefer L1 otherwise, which would cap the CTAs per SM): set as a
+     // launch attribute and, for tools that replay kernels without it (ncu), as the function
+     // attribute of the EPI 0/1 instances — changed only when a launch needs another split
+    size_t pct = 0;
+    if (stage) {
+      const size_t need = (size_t)(2048 / C) * (stage + 2048);
+      pct = (need * 100 + 228 * 1024 - 1) / (228 * 1024);
+      if (pct > 100) pct = 100;
+      attr[1].id = cudaLaunchAttributePreferredSharedMemoryCarveout;
+      attr[1].val.sharedMemCarveout = (unsigned)pct;
+      cfg.numAttrs = 2;
+    }
+    static int set_pct[2] = {0, 0};  // per EPI 0/1 instance of this template; attr_spmv starts at 0
+    const int e = a.epi ? 1 : 0;
+    if (!a.ablate && a.npeer == 0 && set_pct[e] != (int)pct) {
+      if (e) cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 1>, cudaFuncAttributePreferredSharedMemoryCarveout, (int)pct);
+      else cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 0>, cudaFuncAttributePreferredSharedMemoryCarveout, (int)pct);
+      set_pct[e] = (int)pct;
+    }
   }
   // EPI: 0 plain SpMV, 1 power-iteration epilogue, 2 epilogue + peer stores (fused
   // exchange), 3 ablation / roofline probes (h = w = 1 only); separate instances so that
