@@ -195,6 +195,12 @@ __device__ __forceinline__ double ld_relaxed_f64(const double* p) {
 }
 }  // namespace dev
 
+// the launch epoch of this CTA (block-id mode): set by thread 0 at its first tile's scan
+__device__ __forceinline__ unsigned long long& cta_epoch_slot() {
+  __shared__ unsigned long long e;
+  return e;
+}
+
 // Output store.  In a fused exchange (EPI == 2 instances) the element goes to
 // every rank's copy of the next x over peer memory (NVLink P2P stores through IPC
 // mappings; the rank's own buffer is one of them), so the all-gather overlaps the SpMV.
@@ -456,7 +462,10 @@ __device__ __forceinline__ void stream_tile(const KArgs& a, const int64_t tile, 
       cudaTriggerProgrammaticLaunchCompletion();
     }
     if (t == 0) {
-      tk = atomicAdd(a.ticket, 1ull);  // consumed only at the scan barrier (epoch)
+      // one ticket per CTA, advanced by the CTA's tile count (a launch still adds ntiles): the
+      // launch epoch, consumed only at the scan barrier; later tiles of the CTA reuse it
+      const int64_t c0 = (int64_t)blockIdx.x * max(a.tpc, 1);
+      if (tile == c0) tk = atomicAdd(a.ticket, (unsigned long long)(min(a.ntiles, c0 + max(a.tpc, 1)) - c0));
       if constexpr (EPI == 1 || EPI == 2) sh.inv = (a.epi & 1) ? 1.0 / sqrt(a.in_norm2[0]) : 1.0;
     }
   }
@@ -598,7 +607,10 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   }
   // block-id mode (in-order dispatch): the ticket only yields the launch epoch,
   // needed from here on, so its atomic latency hides behind the tile's loads
-  if (a.block_ids && t == 0) sh.epoch = tk / (unsigned long long)a.period + 1ull;
+  if (a.block_ids && t == 0) {  // the CTA's first tile took the ticket (stream_tile)
+    if (tile == (int64_t)blockIdx.x * max(a.tpc, 1)) cta_epoch_slot() = tk / (unsigned long long)a.period + 1ull;
+    sh.epoch = cta_epoch_slot();
+  }
   __syncthreads();
   const unsigned long long epoch = sh.epoch;
   int Fw = 0, Nw = 0, Fall = 0;
@@ -656,7 +668,32 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
 #pragma unroll
     for (int r = 0; r < H; ++r) run[r] = Vex[r];
     bool first = dependent;
-    if (a.seg_row == nullptr) {  // segment k is stacked row k: rows are consecutive
+    if constexpr (H == 1 && (EPI == 0 || EPI == 1)) {
+      if (STG) {  // warp-staged stores: the j-th stop of the thread goes to slot nx + j
+        VT rr = run[0];
+        int j = nx;
+#pragma unroll
+        for (int b = 0; b < T; ++b) {
+          rr = rr + pr[b][0];
+          if ((stops >> b) & 1u) {
+            if (first) {
+              dep[0] = rr;
+              dep_row = seg0;
+            } else {
+              const VT o = EPI == 1 ? rr * invv : rr;
+              wbuf[j] = o;
+              if constexpr (EPI == 1) ssv = fma(o, o, ssv);
+            }
+            first = false;
+            ++j;
+            rr = VT(0);
+          }
+        }
+      }
+    }
+    if (STG) {
+      // done above (H = 1, EPI 0/1 only: STG is false otherwise)
+    } else if (a.seg_row == nullptr) {  // segment k is stacked row k: rows are consecutive
       int64_t row = seg0;
 #pragma unroll
       for (int b = 0; b < T; ++b) {
@@ -674,8 +711,6 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
                 const VT o = (EPI == 1 || EPI == 2) ? run[r] * invv : run[r];
                 if (EPI == 3 && (a.ablate & ABL_NO_YSTORE)) {  // probe: the cost of the y stores
                   if (o == VT(-1.25e-30)) out[row * H + r] = o;
-                } else if (STG) {
-                  wbuf[nx + (int)(row - seg0)] = o;  // the warp's staging slice
                 } else {
                   store_out<VT, EPI>(a, out, row * H + r, o);
                 }
@@ -881,7 +916,10 @@ __device__ __forceinline__ void tile_body_s2(const KArgs& a, const int64_t tile,
 #pragma unroll
     for (int r = 0; r < H; ++r) vx[r] = VT(0);
   }
-  if (a.block_ids && t == 0) sh.epoch = tk / (unsigned long long)a.period + 1ull;
+  if (a.block_ids && t == 0) {  // the CTA's first tile took the ticket (stream_tile)
+    if (tile == (int64_t)blockIdx.x * max(a.tpc, 1)) cta_epoch_slot() = tk / (unsigned long long)a.period + 1ull;
+    sh.epoch = cta_epoch_slot();
+  }
   __syncthreads();
   const unsigned long long epoch = sh.epoch;
   int Fw = 0, Fall = 0;
