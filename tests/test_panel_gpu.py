@@ -216,3 +216,46 @@ def test_tune_and_reencode_keep_the_band():
         _check(csr, _run(A, x), x)
     finally:
         A.free()
+
+
+_CTA_SCRIPT = r"""
+import sys, json, numpy as np, torch
+sys.path.insert(0, %r)
+import synth
+from oracle import ref
+from paper_conf_ppopp_yanlzz14_b200 import Matrix
+out = []
+for far, S in ((1, 3), (2, 1)):
+    csr = synth.circuit_like_rows(0, 300_000, n=300_000, band=8192, n_net=3, net_log2=(12, 16))
+    A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=0, B=8192, R=4096, W=2048,
+                        S=S, T=8, C=128, far=far)
+    x = synth.make_x(csr.n, np.float32, "uniform", 3)
+    y1 = A.spmv(torch.from_numpy(x).cuda()).cpu().numpy()
+    y2 = A.spmv(torch.from_numpy(x).cuda()).cpu().numpy()
+    y_ref, bound = ref.spmv(csr.row_ptr, csr.col, csr.val, x)
+    ok, worst = ref.check_tolerance(y1, y_ref, bound, np.float32)
+    out.append(dict(ok=bool(ok), worst=float(worst), det=bool(np.array_equal(y1.view(np.uint32), y2.view(np.uint32))),
+                    regs=A.info()["band_regs"] if "band_regs" in A.info() else None))
+    A.free()
+print("CTA-RESULT " + json.dumps(out))
+"""
+
+
+@pytest.mark.parametrize("cta", [512, 640, 704, 768, 896, 1024])
+def test_band_kernel_every_cta_size(cta):
+    """The band kernel's CTA size (YASPMV_PANEL_CTA, read once per process): every compiled
+    size — 19 / 21 / 23 / 27 / 31 compute warps + the window producer — against the oracle
+    (separate far part with S = 3, and the far entries as slice 0, P7), run-to-run bitwise."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, YASPMV_PANEL_CTA=str(cta))
+    r = subprocess.run([sys.executable, "-c", _CTA_SCRIPT % root], env=env, capture_output=True, text=True,
+                       timeout=600)
+    line = [l for l in r.stdout.splitlines() if l.startswith("CTA-RESULT ")]
+    assert line, r.stdout[-2000:] + r.stderr[-2000:]
+    for res in json.loads(line[0][len("CTA-RESULT "):]):
+        assert res["ok"], res
+        assert res["det"], res

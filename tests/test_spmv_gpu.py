@@ -340,3 +340,28 @@ def test_warp_staged_stores_bitwise(params, monkeypatch):
     for y in ys[1:]:
         assert np.array_equal(ys[0].view(np.uint32), y.view(np.uint32))
     assert np.array_equal(ys[0].astype(np.float64), exact)
+
+
+def test_warp_staged_stores_power_step(monkeypatch):
+    """The staged stores under the power-iteration epilogue (EPI 1: y scaled by 1/sqrt(in),
+    sum y^2 partials): y and ||y||^2 bitwise equal for wstage 0 and 2 (the per-thread y^2
+    accumulation order is unchanged by the staging)."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix
+    csr = synth.webbase_like(m=60000)
+    x = torch.from_numpy(synth.make_x(csr.n, np.float32, "uniform", 4)).cuda()
+    outs = []
+    for ws in ("0", "2"):
+        monkeypatch.setenv("YASPMV_WSTAGE", ws)
+        A = Matrix.from_csr(csr.m, csr.n, csr.row_ptr, csr.col, csr.val, device=0, T=8, C=128, tpc=2)
+        n_in = torch.full((1,), 4.0, dtype=torch.float64, device="cuda")
+        n_out = torch.zeros(1, dtype=torch.float64, device="cuda")
+        y = torch.empty(csr.m, dtype=torch.float32, device="cuda")
+        A.spmv_power(x, y, n_in, n_out)
+        torch.cuda.synchronize()
+        outs.append((y.cpu().numpy(), float(n_out.item())))
+        A.free()
+    assert np.array_equal(outs[0][0].view(np.uint32), outs[1][0].view(np.uint32))
+    assert outs[0][1] == outs[1][1]
+    y_ref, bound = ref.spmv(csr.row_ptr, csr.col, csr.val, x.cpu().numpy())
+    ok, worst = ref.check_tolerance(outs[0][0], y_ref / 2.0, bound / 2.0, np.float32)
+    assert ok, worst
