@@ -393,6 +393,14 @@ void yaspmv_comm_free(yaspmv_comm c);
 /* ---------------------------------------------------------------- misc */
 const char* yaspmv_last_error(void);
 const char* yaspmv_version(void);
+/* L2 set-aside for persisting accesses on `device` (cudaLimitPersistingL2CacheSize; a
+ * device-wide setting of the calling process — the library never changes it on its own).
+ * The kernels' x gathers are evict_last accesses (the paper's cached x): on C5 the far
+ * part's BCCOO+ slices of x (67 MB at S = 3) keep more of themselves in L2 with a 60 MB
+ * set-aside.  bytes is clamped to the device maximum; *set_bytes (nullable)
+ * receives the value now in effect.  Errors: YASPMV_EINVAL (bad device, bytes < 0),
+ * YASPMV_ECUDA. */
+yaspmv_status yaspmv_l2_persist(int32_t device, int64_t bytes, int64_t* set_bytes);
 /* Per-kernel device timing (measurement only; bench.py's roofline).  yaspmv_profile_begin
  * makes every later SpMV on A record CUDA events on its stream around its kernel groups:
  * stage 0 = the plain BCCOO/BCCOO+ part (K1, + combine, + its y^2 sum), stage 1 = the band

@@ -4,6 +4,6 @@ The product is the C-ABI library ``libyaspmv.so`` (include/yaspmv.h); this packa
 its thin Python binding plus the multi-GPU power-iteration driver (``dist``).
 """
 from ._lib import YaspmvError, EXPORTED  # noqa: F401  (raises ImportError if the .so is missing)
-from .matrix import Comm, Matrix, make_params, nrm2sq, nrm2sq_scratch_bytes, scale, version  # noqa: F401
+from .matrix import Comm, Matrix, l2_persist, make_params, nrm2sq, nrm2sq_scratch_bytes, scale, version  # noqa: F401
 
-__all__ = ["Comm", "Matrix", "make_params", "nrm2sq", "nrm2sq_scratch_bytes", "scale", "version", "YaspmvError"]
+__all__ = ["Comm", "Matrix", "l2_persist", "make_params", "nrm2sq", "nrm2sq_scratch_bytes", "scale", "version", "YaspmvError"]

@@ -761,6 +761,23 @@ extern "C" {
 const char* yaspmv_last_error(void) { return g_err.c_str(); }
 const char* yaspmv_version(void) { return "yaspmv-b200 0.1 (sm_100a)"; }
 
+yaspmv_status yaspmv_l2_persist(int32_t device, int64_t bytes, int64_t* set_bytes) {
+  int ndev = 0;
+  CUDA_TRY(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev || bytes < 0) return fail(YASPMV_EINVAL, "bad device or bytes");
+  DeviceGuard dg(device);
+  int mx = 0;
+  CUDA_TRY(cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, device));
+  const size_t want = (size_t)std::min<int64_t>(bytes, (int64_t)mx);
+  CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+  if (set_bytes) {
+    size_t now = 0;
+    CUDA_TRY(cudaDeviceGetLimit(&now, cudaLimitPersistingL2CacheSize));
+    *set_bytes = (int64_t)now;
+  }
+  return YASPMV_OK;
+}
+
 yaspmv_status yaspmv_build_csr(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                                const void* vals, yaspmv_dtype dtype, const yaspmv_params* params,
                                int32_t device, yaspmv_matrix* out) {

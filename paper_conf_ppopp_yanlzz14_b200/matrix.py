@@ -325,3 +325,11 @@ def scale(src, dst, norm2, stream=None) -> None:
 
 def version() -> str:
     return lib.yaspmv_version().decode()
+
+
+def l2_persist(device: int, nbytes: int) -> int:
+    """cudaLimitPersistingL2CacheSize for `device` (yaspmv_l2_persist): the L2 set-aside the
+    kernels' evict_last x gathers use; returns the bytes now in effect."""
+    out = ctypes.c_int64()
+    check(lib.yaspmv_l2_persist(device, nbytes, ctypes.byref(out)))
+    return out.value

@@ -246,3 +246,19 @@ def test_debug_spin_bound_traps_with_tile_id(tmp_path):
     r = subprocess.run([sys.executable, str(script)], capture_output=True, text=True, timeout=300, env=env)
     assert "TRAPPED" in r.stdout, r.stdout + r.stderr[-2000:]
     assert "SPIN-TILE 2" in r.stdout, r.stdout
+
+
+def test_l2_persist_set_aside():
+    """yaspmv_l2_persist: the set-aside is applied (clamped to the device maximum), SpMV
+    results are bitwise unchanged by it (only cache residency changes), and 0 restores it."""
+    from paper_conf_ppopp_yanlzz14_b200 import Matrix, l2_persist
+    csr = synth.webbase_like(m=50000)
+    x = torch.from_numpy(synth.make_x(csr.n, np.float32, "uniform", 1)).cuda()
+    A = Matrix.from_synth(csr, device=0, T=8, C=128, S=2)
+    y0 = A.spmv(x).cpu().numpy()
+    got = l2_persist(0, 60 << 20)
+    assert got > 0
+    y1 = A.spmv(x).cpu().numpy()
+    assert np.array_equal(y0.view(np.uint32), y1.view(np.uint32))
+    assert l2_persist(0, 0) == 0
+    A.free()
