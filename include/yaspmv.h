@@ -379,13 +379,17 @@ int32_t yaspmv_launches_per_fused_step(yaspmv_matrix A);
  * After bind, yaspmv_comm_x returns the bound buffers and every fused step stores through
  * the multicast mapping.  Errors: YASPMV_EUNSUPPORTED without switch multicast or driver
  * entry points, YASPMV_ECUDA with the CUresult of a failing driver call; a failed sequence
- * leaves the comm on peer stores (mc_active = 0). */
+ * leaves the comm on peer stores (mc_active = 0); if another rank failed, every rank that
+ * did bind calls yaspmv_comm_mc_release (dist.FusedPowerIteration does). */
 int32_t yaspmv_comm_mc_supported(int32_t device);
 yaspmv_status yaspmv_comm_mc_create(yaspmv_comm c, int64_t* fd_out);
 yaspmv_status yaspmv_comm_mc_import(yaspmv_comm c, int64_t pid, int64_t fd);
 yaspmv_status yaspmv_comm_mc_add_device(yaspmv_comm c);
 yaspmv_status yaspmv_comm_mc_bind(yaspmv_comm c);
 int32_t yaspmv_comm_mc_active(yaspmv_comm c);
+/* back to peer stores after a bind (e.g. another rank's bind failed): the x buffers' contents
+ * return to the peer-mapped allocation; the multicast mappings stay until yaspmv_comm_free. */
+yaspmv_status yaspmv_comm_mc_release(yaspmv_comm c);
 /* NULL-safe; unmaps the peers and frees the allocation (synchronize first; peers must not
  * write into this comm any more). */
 void yaspmv_comm_free(yaspmv_comm c);

@@ -40,7 +40,7 @@ EXPORTED = ["yaspmv_build_csr", "yaspmv_build_coo", "yaspmv_free", "yaspmv_spmv"
             "yaspmv_comm_norm2_device", "yaspmv_comm_seq", "yaspmv_comm_check", "yaspmv_launches_per_fused_step",
             "yaspmv_comm_free", "yaspmv_debug_spin_tile", "yaspmv_profile_begin", "yaspmv_profile_end",
             "yaspmv_comm_mc_supported", "yaspmv_comm_mc_create", "yaspmv_comm_mc_import",
-            "yaspmv_comm_mc_add_device", "yaspmv_comm_mc_bind", "yaspmv_comm_mc_active", "yaspmv_l2_persist",
+            "yaspmv_comm_mc_add_device", "yaspmv_comm_mc_bind", "yaspmv_comm_mc_active", "yaspmv_comm_mc_release", "yaspmv_l2_persist",
             # include/yaspmv_ablation.h
             "yaspmv_ablation_spmv", "yaspmv_ablation_tree", "yaspmv_ablation_tree_scratch_bytes"]
 
@@ -138,6 +138,7 @@ def _load():
         "yaspmv_comm_mc_add_device": ([H], ctypes.c_int),
         "yaspmv_comm_mc_bind": ([H], ctypes.c_int),
         "yaspmv_comm_mc_active": ([H], i32),
+        "yaspmv_comm_mc_release": ([H], ctypes.c_int),
         "yaspmv_l2_persist": ([i32, i64, ctypes.POINTER(i64)], ctypes.c_int),
         "yaspmv_debug_spin_tile": ([], i64),
         "yaspmv_profile_begin": ([H], ctypes.c_int),

@@ -442,6 +442,17 @@ yaspmv_status yaspmv_comm_mc_bind(yaspmv_comm c) {
 
 int32_t yaspmv_comm_mc_active(yaspmv_comm c) { return c && c->mc ? 1 : 0; }
 
+yaspmv_status yaspmv_comm_mc_release(yaspmv_comm c) {
+  if (!c) return fail(YASPMV_EINVAL, "NULL comm");
+  if (c->mc) {  // back to the peer-mapped buffers (the bound ones stay mapped until free)
+    CUDA_TRY(cudaSetDevice(c->device));
+    CUDA_TRY(cudaDeviceSynchronize());
+    CUDA_TRY(cudaMemcpy(c->base, reinterpret_cast<void*>(c->loc_va), 2 * c->xbytes, cudaMemcpyDeviceToDevice));
+    c->mc = false;
+  }
+  return YASPMV_OK;
+}
+
 yaspmv_status yaspmv_comm_begin(yaspmv_comm c) {
   if (!c) return fail(YASPMV_EINVAL, "NULL comm");
   c->fresh = true;

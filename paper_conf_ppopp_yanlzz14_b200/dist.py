@@ -271,6 +271,10 @@ class FusedPowerIteration:
             stage(comm.mc_add_device, "add the devices to the multicast object")
             stage(comm.mc_bind, "bind the x buffers to the multicast object")
         except RuntimeError:
+            # every rank learned of the failure (the stages are agreed on): a rank whose own
+            # bind succeeded goes back to peer stores too, so all ranks use one protocol
+            if getattr(comm, "mc_active", False):
+                comm.mc_release()
             if required:
                 raise
         self.multicast = bool(getattr(comm, "mc_active", False))

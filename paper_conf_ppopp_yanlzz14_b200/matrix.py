@@ -254,6 +254,9 @@ class Comm:
     def mc_active(self) -> bool:
         return bool(lib.yaspmv_comm_mc_active(self._h))
 
+    def mc_release(self) -> None:
+        check(lib.yaspmv_comm_mc_release(self._h))
+
     def x(self, which: int = 0):
         """torch view of x buffer (seq + which) % 2 (which = 0: the next step's input /
         the latest z; 1: the buffer the next step writes), world * chunk elements."""

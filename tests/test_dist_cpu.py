@@ -308,3 +308,96 @@ def test_fused_setup_failure_is_agreed_by_every_rank(mode):
     want = {"create": "create the exchange buffers on rank(s) [0]", "open": "map the peers' buffers on rank(s) [1]",
             "handle": "export the IPC handles on rank(s) [1]"}[mode]
     assert all(want in o for o in outs), outs
+
+
+# ---------------------------------------------------------------- multicast setup (host side)
+class _McShmComm(_ShmComm):
+    """The multicast setup calls of yaspmv_comm_mc_* on the shared-file comm: each call is
+    logged; ``fail`` names a stage that raises on rank 1.  A bound comm keeps the peer-store
+    protocol of _ShmComm underneath (the exchange itself is modelled by the parent)."""
+
+    fail = None
+
+    def __init__(self, *a, **kw):
+        super().__init__(*a, **kw)
+        self.log, self.mc_active = [], False
+
+    def _maybe_fail(self, stage):
+        self.log.append(stage)
+        if self.rank == 1 and self.fail == stage:
+            raise OSError(f"{stage} refused on rank 1")
+
+    def mc_supported(self, device):
+        self._maybe_fail("probe")
+        return True
+
+    def mc_create(self):
+        assert self.rank == 0
+        self._maybe_fail("create")
+        return 17
+
+    def mc_import(self, pid, fd):
+        assert fd == 17 and pid > 0 and pid != os.getpid()  # the creator's descriptor
+        self._maybe_fail("import")
+
+    def mc_add_device(self):
+        self._maybe_fail("add")
+
+    def mc_bind(self):
+        self._maybe_fail("bind")
+        self.mc_active = True
+
+    def mc_release(self):
+        self.log.append("release")
+        self.mc_active = False
+
+
+def _mc_worker(rank, world, port, root, fail, multicast):
+    import json
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ["SHM_ROOT"] = root
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n = 1 << 10
+    from synth import matrices as sm
+    full = sm.circuit_like_rows(0, n, n=n, n_net=1, net_log2=(6, 7), band=64)
+    L = D.make_layout(full.row_ptr, rank, world)
+
+    class F(_McShmComm):
+        pass
+    F.fail = fail
+    out = {}
+    try:
+        pit = D.FusedPowerIteration(L, None, torch.float64, "cpu", comm_factory=F, multicast=multicast)
+        out = {"ok": True, "multicast": pit.multicast, "log": pit.comm.log}
+    except RuntimeError as e:
+        out = {"ok": False, "err": str(e)}
+    with open(os.path.join(root, f"mc{rank}.json"), "w") as f:
+        json.dump(out, f)
+    dist.barrier()  # every rank got here: no rank waits on a peer's setup
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("fail,multicast", [(None, True), ("bind", "auto"), ("import", "auto"),
+                                            ("probe", "auto"), ("add", True)])
+def test_multicast_setup_is_agreed_by_every_rank(fail, multicast):
+    """dist.FusedPowerIteration(multicast=...) over gloo world 2: rank 0 creates the object,
+    rank 1 imports rank 0's (pid, fd), both add their device, then bind — every stage agreed
+    on, so a failure anywhere leaves EVERY rank on peer stores (multicast="auto": a rank whose
+    own bind succeeded releases it) or makes every rank raise (multicast=True); no rank hangs."""
+    import json
+    import torch.multiprocessing as mp
+    with tempfile.TemporaryDirectory() as td:
+        mp.spawn(_mc_worker, args=(2, _free_port(), td, fail, multicast), nprocs=2, join=True)
+        res = [json.load(open(os.path.join(td, f"mc{r}.json"))) for r in range(2)]
+    if fail is None:
+        assert all(r["ok"] and r["multicast"] for r in res)
+        assert res[0]["log"] == ["probe", "create", "add", "bind"]
+        assert res[1]["log"] == ["probe", "import", "add", "bind"]
+    elif multicast is True:
+        assert all(not r["ok"] and "rank(s) [1]" in r["err"] for r in res)
+    else:
+        assert all(r["ok"] and not r["multicast"] for r in res)
+        if fail == "bind":  # rank 0 had bound: it went back to peer stores
+            assert res[0]["log"][-1] == "release"
