@@ -280,14 +280,17 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     // the low 16 bits and the has-stop flag above (a sum of flags is non-zero iff their OR is)
     int fn_ = nst | ((nst > 0) << 16);
     VT v = tail;
-    if (__ballot_sync(0xffffffffu, nst > 0) == 0xffffffffu) {
+    const bool allstop = __ballot_sync(0xffffffffu, nst > 0) == 0xffffffffu;
+    int nx_fast = 0;
+    if (allstop) {
       // every lane holds a stop (the common case): each lane's scanned value is its own
-      // tail, only the stop counts need the scan (the skip of P:222 at thread level)
+      // tail (the skip of P:222 at thread level), and the stops of the earlier lanes are
+      // counted by bit planes of the per-lane counts (nst <= 16: five ballots + popc, no
+      // shuffle chain)
+      const unsigned ltm = (1u << lane) - 1u;
 #pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const int g2 = __shfl_up_sync(0xffffffffu, fn_, d);
-        if (lane >= d) fn_ += g2 & 0xFFFF;
-      }
+      for (int b = 0; b < 5; ++b) nx_fast += __popc(__ballot_sync(0xffffffffu, (nst >> b) & 1) & ltm) << b;
+      fn_ = (nx_fast + nst) | (1 << 16);
     } else {
 #pragma unroll
       for (int d = 1; d < 32; d <<= 1) {
@@ -311,15 +314,17 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       sh.rtag[lt % RING] = 2 * (lt + 1) + (final_now ? 1 : 0);
     }
     prefetch();  // the warp's next tile in flight during this tile's updates and look-back
-    const int gx = __shfl_up_sync(0xffffffffu, fn_, 1);
-    int fx = (gx >> 16) != 0;
-    int nx = gx & 0xFFFF;
-    VT vx = __shfl_up_sync(0xffffffffu, v, 1);
-    if (lane == 0) {
-      fx = 0;
-      nx = 0;
-      vx = VT(0);
+    int fx, nx;
+    if (allstop) {
+      fx = lane > 0;
+      nx = nx_fast;
+    } else {
+      const int gx = __shfl_up_sync(0xffffffffu, fn_, 1);
+      fx = lane > 0 && (gx >> 16) != 0;
+      nx = lane > 0 ? gx & 0xFFFF : 0;
     }
+    VT vx = __shfl_up_sync(0xffffffffu, v, 1);
+    if (lane == 0) vx = VT(0);
     if (pending) {  // every warp is done with slice o - 1 (acc order)
       slice_barrier(o);
       pending = false;
@@ -360,7 +365,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     // walk stops at, so y is bitwise deterministic.  Needed by the warp's first stop (dep)
     // and, for a tile without a stop, by its own carry-out (a row spanning many tiles walks
     // O(warps) records per tile, not O(its length))
-    const bool nostop = !__shfl_sync(0xffffffffu, f, 31);
+    const bool nostop = !allstop && !__shfl_sync(0xffffffffu, f, 31);
     const unsigned dball = __ballot_sync(0xffffffffu, dep);
     if (dball || (nostop && u > 0)) {
       VT carry = VT(0);
