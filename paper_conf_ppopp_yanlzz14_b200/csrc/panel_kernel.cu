@@ -37,6 +37,9 @@ namespace yaspmv {
 namespace {
 
 constexpr int BT = PANEL_BT;
+#ifndef PANEL_ACC_RUN
+#define PANEL_ACC_RUN 4  // positions per acc update chain (BT / RUN chains, RUN rounds)
+#endif
 
 __device__ __forceinline__ uint64_t pol_evict_first() {
   uint64_t p;
@@ -341,19 +344,27 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
       // 4q..4q+3 own the rows from row_first + the stops before 4q on): their loads issue
       // back to back instead of one shared-memory round trip per stop; the chains touch
       // disjoint rows, so the result is the same as the sequential walk
-      static_assert(BT == 16, "four chains of four positions");
-      const int c1 = __popc(stops & 0xFu), c2 = c1 + __popc(stops & 0xF0u), c3 = c2 + __popc(stops & 0xF00u);
-      VT* aq[4] = {acc + row_first, acc + row_first + c1, acc + row_first + c2, acc + row_first + c3};
+      static_assert(BT == 16, "chains of PANEL_ACC_RUN positions");
+      constexpr int RUN = PANEL_ACC_RUN, NQ = BT / RUN;
+      VT* aq[NQ];
+      {
+        int c = 0;
 #pragma unroll
-      for (int r = 0; r < 4; ++r) {
-        VT l[4];
+        for (int q = 0; q < NQ; ++q) {
+          aq[q] = acc + row_first + c;
+          c += __popc(stops & (((1u << RUN) - 1u) << (RUN * q)));
+        }
+      }
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if ((stops >> (4 * q + r)) & 1u) l[q] = *aq[q];
+      for (int r = 0; r < RUN; ++r) {
+        VT l[NQ];
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if ((stops >> (4 * q + r)) & 1u) {
-            *aq[q] = l[q] + pr[4 * q + r];
+        for (int q = 0; q < NQ; ++q)
+          if ((stops >> (RUN * q + r)) & 1u) l[q] = *aq[q];
+#pragma unroll
+        for (int q = 0; q < NQ; ++q)
+          if ((stops >> (RUN * q + r)) & 1u) {
+            *aq[q] = l[q] + pr[RUN * q + r];
             ++aq[q];
           }
       }
