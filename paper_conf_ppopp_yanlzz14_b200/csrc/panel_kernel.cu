@@ -454,10 +454,18 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
   };
   // this warp's first tile in slice kk or a later non-empty slice that has one: its
   // panel-local tile index, -1 if none
+  // Tiles go to the compute warps round-robin over the panel's whole tile sequence (tile lt
+  // to warp lt mod NCW, continuing across slice boundaries), not restarting at warp 0 in
+  // every slice: the warps that finish slice o first take slice o+1's first tiles, so the
+  // per-slice remainder does not pile up on the same warps (balance at the slice barriers)
+  auto first_u = [&](int kk) {  // this warp's first slice-local tile index in slice kk
+    const int l0 = sh.sp[kk] >> 9;
+    return (wid - l0 % NCW + NCW) % NCW;
+  };
   auto first_tile_from = [&](int kk) {
     kk = next_nonempty(kk);
-    while (kk < KS && (sh.sp[kk + 1] - sh.sp[kk]) >> 9 <= wid) kk = next_nonempty(kk + 1);
-    return kk < KS ? (sh.sp[kk] >> 9) + wid : -1;
+    while (kk < KS && (sh.sp[kk + 1] - sh.sp[kk]) >> 9 <= first_u(kk)) kk = next_nonempty(kk + 1);
+    return kk < KS ? (sh.sp[kk] >> 9) + first_u(kk) : -1;
   };
   if (k < KS) {  // the warp's first band tile in flight before the first window wait
     const int f = first_tile_from(k);
@@ -475,7 +483,7 @@ __global__ void __launch_bounds__(NTH, 1) panel_kernel(const PanelArgs a) {
     const VT* wk = win(ow) + shift_of(k);
     const int frk = sh.fr[k];
     bool pending = o > 0;  // X_o still ahead of this warp
-    for (int u = wid; u < ntile_k; u += NCW) {
+    for (int u = first_u(k); u < ntile_k; u += NCW) {
       const int lt = ltile_k + u;       // panel-local tile index (tag of its carry record)
       flow(lt, u, ntile_k);
       // ---- multiply: gathers from the slice's window --------------------------------
