@@ -283,7 +283,7 @@ yaspmv_status resolve_band(yaspmv_matrix A, Params& p) {
   if (p.bfar != YASPMV_FAR_SEPARATE && p.bfar != YASPMV_FAR_IN_PANEL) return fail(YASPMV_EINVAL, "bad band_far");
   if (A->dtype != YASPMV_F32) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ is compiled for fp32");
   if (p.h != 1 || p.w != 1) return fail(YASPMV_EUNSUPPORTED, "panel-sliced BCCOO+ needs 1x1 blocks");
-  if (p.pR == 0) p.pR = 16384;  // defaults: one 1024-thread CTA per SM, 205 KB of shared memory
+  if (p.pR == 0) p.pR = 16384;  // defaults: one CTA per SM (PANEL_CTA threads), ~200 KB of shared memory
   if (p.pW == 0) p.pW = 16384;
   if (p.pR % 256 || p.pR <= 0 || p.pR > 32768) return fail(YASPMV_EINVAL, "panel_rows must be a multiple of 256 in [256, 32768]");
   if (p.pW % 4 || p.pW <= 0 || p.pW > 65532) return fail(YASPMV_EINVAL, "slice_width must be a multiple of 4 in [4, 65532]");
