@@ -587,8 +587,10 @@ yaspmv_status run_spmv_plain(yaspmv_matrix A, const void* x, void* y, void* stre
      // (C5: one scattered 4-byte store per row made a third of the far kernel's L2 requests;
      // staged + streaming stores: 1.25 -> 1.13 ms); YASPMV_WSTAGE = 0 / 1 / 2 overrides
     const char* e = std::getenv("YASPMV_WSTAGE");
-    const int want = e ? std::atoi(e) : (A->band_on ? 2 : 0);
-    a.wstage = (want && p.h == 1 && p.rc == 0 && !ablate && !(peers && p.S == 1) && c.n_zero == 0 &&
+    // (also on for the fused exchange's peer stores: each warp's rows go to every peer as
+    // contiguous runs instead of P scattered stores per row)
+    const int want = e ? std::atoi(e) : ((A->band_on || peers) ? 2 : 0);
+    a.wstage = (want && p.h == 1 && p.rc == 0 && !ablate && c.n_zero == 0 &&
                 A->d.seg_row == nullptr && (int64_t)p.C * p.T * A->vsize <= 40 * 1024)
                    ? want
                    : 0;

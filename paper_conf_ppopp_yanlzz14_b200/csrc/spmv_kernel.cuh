@@ -527,7 +527,8 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
   VT* out = static_cast<VT*>(a.out);
   // warp-staged y stores (KArgs::wstage): this warp's slice of the dynamic shared memory
   extern __shared__ __align__(16) unsigned char s1_stage[];
-  VT* const wbuf = (H == 1 && (EPI == 0 || EPI == 1) && a.wstage && a.seg_row == nullptr)
+  // (not in the T = 32 peer-store instance: its registers would spill)
+  VT* const wbuf = (H == 1 && (EPI == 0 || EPI == 1 || (EPI == 2 && T <= 16)) && a.wstage && a.seg_row == nullptr)
                        ? reinterpret_cast<VT*>(s1_stage) + wid * 32 * T
                        : nullptr;
   const bool STG = wbuf != nullptr;
@@ -668,7 +669,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
 #pragma unroll
     for (int r = 0; r < H; ++r) run[r] = Vex[r];
     bool first = dependent;
-    if constexpr (H == 1 && (EPI == 0 || EPI == 1)) {
+    if constexpr (H == 1 && (EPI == 0 || EPI == 1 || (EPI == 2 && T <= 16))) {
       if (STG) {  // warp-staged stores: the j-th stop of the thread goes to slot nx + j
         VT rr = run[0];
         int j = nx;
@@ -680,9 +681,9 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
               dep[0] = rr;
               dep_row = seg0;
             } else {
-              const VT o = EPI == 1 ? rr * invv : rr;
+              const VT o = (EPI == 1 || EPI == 2) ? rr * invv : rr;
               wbuf[j] = o;
-              if constexpr (EPI == 1) ssv = fma(o, o, ssv);
+              if constexpr (EPI == 1 || EPI == 2) ssv = fma(o, o, ssv);
             }
             first = false;
             ++j;
@@ -757,7 +758,7 @@ __device__ __forceinline__ void tile_body(const KArgs& a, const int64_t tile, Sc
     const int wcnt = __shfl_sync(0xffffffffu, nn, 31);
     const int skip = __ballot_sync(0xffffffffu, dependent) != 0u;  // slot 0: the carried segment
     const int64_t wrow0 = (int64_t)cta_seg0 + Nw;
-    if (a.wstage == 2) {  // streaming stores (the slice results are read by a later kernel)
+    if (EPI != 2 && a.wstage == 2) {  // streaming stores (the slice results are read by a later kernel)
       for (int i = lane + skip; i < wcnt; i += 32) __stcs(out + wrow0 + i, wbuf[i]);
     } else {
       for (int i = lane + skip; i < wcnt; i += 32) store_out<VT, EPI>(a, out, wrow0 + i, wbuf[i]);
@@ -1069,10 +1070,11 @@ void launch_spmv(const KArgs& a, int C, int64_t grid, void* stream) {
       attr[1].val.sharedMemCarveout = (unsigned)pct;
       cfg.numAttrs = 2;
     }
-    static int set_pct[2] = {0, 0};  // per EPI 0/1 instance of this template; attr_spmv starts at 0
-    const int e = a.epi ? 1 : 0;
-    if (!a.ablate && a.npeer == 0 && set_pct[e] != (int)pct) {
-      if (e) cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 1>, cudaFuncAttributePreferredSharedMemoryCarveout, (int)pct);
+    static int set_pct[3] = {0, 0, 0};  // per EPI 0/1/2 instance of this template; attr_spmv starts at 0
+    const int e = a.npeer > 0 ? 2 : a.epi ? 1 : 0;
+    if (!a.ablate && set_pct[e] != (int)pct) {
+      if (e == 2) cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 2>, cudaFuncAttributePreferredSharedMemoryCarveout, (int)pct);
+      else if (e) cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 1>, cudaFuncAttributePreferredSharedMemoryCarveout, (int)pct);
       else cudaFuncSetAttribute(spmv_bccoo_kernel<VT, H, W, T, CM, 0>, cudaFuncAttributePreferredSharedMemoryCarveout, (int)pct);
       set_pct[e] = (int)pct;
     }
@@ -1110,6 +1112,8 @@ int attr_spmv(int C, int /*rc*/, int* regs, int* max_threads, int* blocks_per_sm
     e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, max((int)TR::smem_bytes(C), stage_cap));
     if (e != cudaSuccess) return (int)e;
     e = cudaFuncSetAttribute(k2, cudaFuncAttributeMaxDynamicSharedMemorySize, max((int)TR::smem_bytes(C), stage_cap));
+    if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize, max((int)TR::smem_bytes(C), stage_cap));
     if (e != cudaSuccess) return (int)e;
     // x gathers are the L1 traffic: give L1 the whole unified carve-out
     e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 0);
