@@ -520,9 +520,25 @@ def main():
         # the fused exchange (SpMV epilogue stores z into every rank's x; no NCCL), with peer
         # stores and, where the GPUs report switch multicast, with one multimem.st per element
         fused_info = {}
+
+        def agreed_check(comm):
+            # every rank learns whether any rank's device waits timed out, and all raise
+            # together (no rank is left in a collective the others skipped)
+            ok = 1
+            try:
+                comm.check()
+            except Exception:
+                ok = 0
+            t = torch.tensor([ok], dtype=torch.int32, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN)
+            if int(t.item()) == 0:
+                raise RuntimeError("a fused step's device wait timed out on some rank")
+
         for mode, mc in (("p2p", False), ("multicast", "auto")):
             try:
-                fp = D.FusedPowerIteration(L, A, tdt, dev, timeout_ms=20000, multicast=mc)
+                # a short device-wait timeout: a peer signal that never arrives costs seconds,
+                # not minutes, and the warm-up check below skips the timed loop
+                fp = D.FusedPowerIteration(L, A, tdt, dev, timeout_ms=5000, multicast=mc)
                 if mc and not fp.multicast:
                     fused_info[mode] = {"unavailable": "no switch multicast on every rank"}
                     dist.barrier()
@@ -532,6 +548,7 @@ def main():
                     fp.step(stream)
                 fp.comm.wait(stream)
                 torch.cuda.synchronize()
+                agreed_check(fp.comm)  # a warm-up step timed out on any rank: all skip the timed loop
                 dist.barrier()
                 f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 f0.record(stream)
@@ -540,7 +557,7 @@ def main():
                 fp.comm.wait(stream)
                 f1.record(stream)
                 torch.cuda.synchronize()
-                fp.comm.check()
+                agreed_check(fp.comm)
                 tf = torch.tensor([f0.elapsed_time(f1) / 20], dtype=torch.float64, device=dev)
                 dist.all_reduce(tf, op=dist.ReduceOp.MAX)
                 fused_info[mode] = {"ms_per_step": float(tf.item()), "steps": 20,
